@@ -1,0 +1,263 @@
+"""B200-native chunked LZ compression (Ma & Park, PaCT 2017 -- the GPU side of
+inline compression of fixed-size write chunks).
+
+Thin Python binding over the C ABI of ``liblzr.so`` (``include/lzr.h``):
+argument marshalling only.  Every step of the path (staging, match search,
+greedy token selection, encoding, scan, compaction, decoding) runs in the
+sm_100a kernels of ``csrc/``.  PyTorch is used for device memory and streams.
+There is no CPU fallback: importing this package fails loudly when the CUDA
+library has not been built, and the compute calls need a CUDA device.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+__all__ = [
+    "Params", "LzrError", "lib", "num_chunks", "compress_bound", "compress_workspace_bytes",
+    "compress", "compress_encode", "compress_compact", "scan_sizes", "decompress",
+    "compress_host", "validate_params", "status_str", "last_launch_count",
+]
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "liblzr.so")
+
+OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CAPACITY, ERR_CUDA, ERR_CORRUPT = 0, -1, -2, -3, -4, -5
+
+EXPORTED_SYMBOLS = [
+    "lzr_validate_params", "lzr_num_chunks", "lzr_compress_bound", "lzr_compress_workspace_bytes",
+    "lzr_compress_chunks", "lzr_compress_encode", "lzr_compress_compact",
+    "lzr_scan_workspace_bytes", "lzr_scan_sizes", "lzr_decompress_chunks",
+    "lzr_compress_host_scratch_bytes", "lzr_compress_host", "lzr_status_str",
+    "lzr_last_launch_count",
+]
+
+
+class LzrError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        super().__init__(f"{what}: {status_str(status)} ({status})")
+        self.status = status
+
+
+class _CParams(ctypes.Structure):
+    _fields_ = [("chunk_size", ctypes.c_uint32), ("window", ctypes.c_uint32),
+                ("min_match", ctypes.c_uint32), ("max_match", ctypes.c_uint32),
+                ("tie_break", ctypes.c_uint32)]
+
+
+@dataclass(frozen=True)
+class Params:
+    """lzr_params.  Defaults: C = W = 4096, m = 4, M = m + 255 (R1-R7)."""
+    chunk_size: int = 4096
+    window: int | None = None
+    min_match: int = 4
+    max_match: int | None = None
+    tie_break: int = 0
+
+    def c(self) -> _CParams:
+        w = self.chunk_size if self.window is None else self.window
+        mm = self.min_match + 255 if self.max_match is None else self.max_match
+        return _CParams(self.chunk_size, w, self.min_match, mm, self.tie_break)
+
+
+_lib = None
+
+
+def lib():
+    """Load liblzr.so.  Raises if it has not been built (no fallback path)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(
+                f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; "
+                "g.build()'` (nvcc, sm_100a).  There is no CPU fallback.")
+        L = ctypes.CDLL(LIB_PATH)
+        P = ctypes.POINTER(_CParams)
+        vp, sz, u64 = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_uint64
+        L.lzr_validate_params.argtypes = [P]
+        L.lzr_num_chunks.argtypes = [sz, P]
+        L.lzr_num_chunks.restype = sz
+        L.lzr_compress_bound.argtypes = [sz, P]
+        L.lzr_compress_bound.restype = sz
+        L.lzr_compress_workspace_bytes.argtypes = [sz, P]
+        L.lzr_compress_workspace_bytes.restype = sz
+        L.lzr_compress_chunks.argtypes = [vp, sz, P, vp, sz, vp, vp, vp, vp, sz, vp]
+        L.lzr_compress_encode.argtypes = [vp, sz, P, vp, vp, sz, vp]
+        L.lzr_compress_compact.argtypes = [vp, sz, P, vp, sz, vp, vp, vp, vp, sz, vp]
+        L.lzr_scan_workspace_bytes.argtypes = [sz]
+        L.lzr_scan_workspace_bytes.restype = sz
+        L.lzr_scan_sizes.argtypes = [vp, sz, u64, vp, vp, vp, sz, vp]
+        L.lzr_decompress_chunks.argtypes = [vp, vp, vp, sz, P, vp, vp, vp]
+        L.lzr_compress_host_scratch_bytes.argtypes = [sz, P]
+        L.lzr_compress_host_scratch_bytes.restype = sz
+        L.lzr_compress_host.argtypes = [vp, sz, P, vp, sz, vp, vp, vp, sz, vp, sz]
+        L.lzr_status_str.argtypes = [ctypes.c_int]
+        L.lzr_status_str.restype = ctypes.c_char_p
+        L.lzr_last_launch_count.argtypes = []
+        _lib = L
+    return _lib
+
+
+def status_str(st: int) -> str:
+    return lib().lzr_status_str(st).decode()
+
+
+def _check(st: int, what: str):
+    if st != OK:
+        raise LzrError(st, what)
+
+
+def validate_params(p: Params) -> int:
+    return lib().lzr_validate_params(ctypes.byref(p.c()))
+
+
+def num_chunks(n: int, p: Params) -> int:
+    return lib().lzr_num_chunks(n, ctypes.byref(p.c()))
+
+
+def compress_bound(n: int, p: Params) -> int:
+    return lib().lzr_compress_bound(n, ctypes.byref(p.c()))
+
+
+def compress_workspace_bytes(n: int, p: Params) -> int:
+    return lib().lzr_compress_workspace_bytes(n, ctypes.byref(p.c()))
+
+
+def last_launch_count() -> int:
+    return lib().lzr_last_launch_count()
+
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr() if t is not None and t.numel() else 0)
+
+
+def _stream(stream, device):
+    import torch
+
+    s = stream if stream is not None else torch.cuda.current_stream(device)
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _require_cuda_u8(t, name):
+    import torch
+
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.uint8 and t.is_contiguous()):
+        raise TypeError(f"{name} must be a contiguous uint8 CUDA tensor")
+
+
+class Workspace:
+    """Reusable device buffers for repeated compress() calls of one size."""
+
+    def __init__(self, n: int, p: Params, device=None):
+        import torch
+
+        self.n, self.p = n, p
+        dev = torch.device(device) if device is not None else torch.device("cuda")
+        N = num_chunks(n, p)
+        self.out = torch.empty(max(1, compress_bound(n, p)), dtype=torch.uint8, device=dev)
+        self.sizes = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+        self.offsets = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+        self.total = torch.zeros(1, dtype=torch.int64, device=dev)
+        self.ws = torch.empty(max(256, compress_workspace_bytes(n, p)), dtype=torch.uint8, device=dev)
+        self.N = N
+
+
+def compress(t, p: Params = Params(), ws: Workspace | None = None, stream=None):
+    """Compress a uint8 CUDA tensor chunk by chunk.
+
+    Returns (out, sizes, offsets, total): ``out`` holds ``capacity = n`` bytes of
+    which the first ``total`` are the compacted chunk streams; ``sizes`` int32
+    (bit pattern of the ABI's uint32), ``offsets`` int64, ``total`` int64[1] --
+    all device tensors; nothing is synchronised.
+    """
+    _require_cuda_u8(t, "input")
+    n = t.numel()
+    if ws is None or ws.n != n or ws.p != p:
+        ws = Workspace(n, p, t.device)
+    st = lib().lzr_compress_chunks(
+        _ptr(t), n, ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
+        _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    _check(st, "lzr_compress_chunks")
+    N = ws.N
+    return ws.out, ws.sizes[:N], ws.offsets[:N], ws.total
+
+
+def compress_encode(t, p: Params, ws: Workspace, stream=None):
+    """Launch only the encode stage (bench timing): sizes in ws.sizes."""
+    st = lib().lzr_compress_encode(_ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.sizes),
+                                   _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    _check(st, "lzr_compress_encode")
+
+
+def compress_compact(t, p: Params, ws: Workspace, stream=None):
+    """Launch only the scan + compaction stage (after compress_encode)."""
+    st = lib().lzr_compress_compact(
+        _ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
+        _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    _check(st, "lzr_compress_compact")
+
+
+def scan_sizes(sizes, base: int = 0, offsets=None, total=None, ws=None, stream=None):
+    """Exclusive prefix sum (+ base) of int32/uint32 sizes on the device."""
+    import torch
+
+    n = sizes.numel()
+    if offsets is None:
+        offsets = torch.empty(max(1, n), dtype=torch.int64, device=sizes.device)
+    if total is None:
+        total = torch.zeros(1, dtype=torch.int64, device=sizes.device)
+    wsb = lib().lzr_scan_workspace_bytes(n)
+    if ws is None or ws.numel() < wsb:
+        ws = torch.empty(max(256, wsb), dtype=torch.uint8, device=sizes.device)
+    st = lib().lzr_scan_sizes(_ptr(sizes), n, base, _ptr(offsets), _ptr(total), _ptr(ws),
+                              ws.numel(), _stream(stream, sizes.device))
+    _check(st, "lzr_scan_sizes")
+    return offsets[:n], total
+
+
+def decompress(comp, sizes, offsets, n: int, p: Params = Params(), out=None, error=None,
+               stream=None):
+    """Decode chunk streams back into n bytes.  Returns (out, error) where
+    error is an int32[1] device tensor: 0 or 1 + index of the first corrupt chunk."""
+    import torch
+
+    dev = comp.device
+    if out is None:
+        out = torch.empty(max(1, n), dtype=torch.uint8, device=dev)
+    if error is None:
+        error = torch.zeros(1, dtype=torch.int32, device=dev)
+    st = lib().lzr_decompress_chunks(_ptr(comp), _ptr(sizes), _ptr(offsets), n,
+                                     ctypes.byref(p.c()), _ptr(out), _ptr(error),
+                                     _stream(stream, dev))
+    _check(st, "lzr_decompress_chunks")
+    return out[:n], error
+
+
+def compress_host(h_in, p: Params = Params(), batch_bytes: int = 0, scratch=None, h_out=None,
+                  h_sizes=None, h_offsets=None):
+    """End-to-end compression of a host (preferably pinned) uint8 tensor through
+    the C ABI's host-buffer pipeline (H2D, kernels, D2H inside).  Synchronous.
+    Returns (h_out, h_sizes, h_offsets, total) on the host."""
+    import torch
+
+    n = h_in.numel()
+    N = num_chunks(n, p)
+    if batch_bytes == 0:
+        batch_bytes = max(p.chunk_size, -(-n // p.chunk_size) * p.chunk_size)
+    need = lib().lzr_compress_host_scratch_bytes(batch_bytes, ctypes.byref(p.c()))
+    if scratch is None or scratch.numel() < need:
+        scratch = torch.empty(max(256, need), dtype=torch.uint8, device="cuda")
+    if h_out is None:
+        h_out = torch.empty(max(1, n), dtype=torch.uint8, pin_memory=True)
+    if h_sizes is None:
+        h_sizes = torch.empty(max(1, N), dtype=torch.int32, pin_memory=True)
+    if h_offsets is None:
+        h_offsets = torch.empty(max(1, N), dtype=torch.int64, pin_memory=True)
+    tot = ctypes.c_uint64()
+    st = lib().lzr_compress_host(
+        ctypes.c_void_p(h_in.data_ptr()), n, ctypes.byref(p.c()), ctypes.c_void_p(h_out.data_ptr()),
+        h_out.numel(), ctypes.c_void_p(h_sizes.data_ptr()), ctypes.c_void_p(h_offsets.data_ptr()),
+        ctypes.byref(tot), batch_bytes, _ptr(scratch), scratch.numel())
+    _check(st, "lzr_compress_host")
+    return h_out, h_sizes[:N], h_offsets[:N], tot.value

@@ -1,0 +1,354 @@
+// capi.cu -- the extern "C" boundary of liblzr.so (include/lzr.h): parameter
+// validation, workspace sizing, launch sequencing on the caller's stream, and
+// the host-buffer end-to-end pipeline.  No device memory is allocated here.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "lzr_internal.cuh"
+
+namespace lzr {
+
+namespace {
+
+struct DevInfo {
+  int sm_count = 0;
+  int smem_optin = 0;
+};
+
+thread_local int t_launches = 0;
+std::mutex g_mu;
+DevInfo g_dev[64];
+
+cudaError_t dev_info(DevInfo* out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (g_dev[dev].sm_count == 0) {
+    int sms = 0, smem = 0;
+    e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess) return e;
+    e = cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    if (e != cudaSuccess) return e;
+    g_dev[dev].sm_count = sms;
+    g_dev[dev].smem_optin = smem;
+  }
+  *out = g_dev[dev];
+  return cudaSuccess;
+}
+
+bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+}  // namespace
+
+WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
+  WsLayout w;
+  const size_t C = p->chunk_size;
+  const size_t N = (n_bytes + C - 1) / C;
+  w.ctrl_off = 0;
+  w.slots_off = 256;
+  w.scan_off = w.slots_off + align_up_z(N * C, 256);
+  w.total = w.scan_off + scan_ws_bytes(N);
+  return w;
+}
+
+}  // namespace lzr
+
+using namespace lzr;
+
+extern "C" {
+
+int lzr_validate_params(const lzr_params* p) {
+  if (!p) return LZR_ERR_INVALID_ARG;
+  if (p->chunk_size < 16 || p->chunk_size > 65536 || p->chunk_size % 16) return LZR_ERR_INVALID_ARG;
+  if (p->window < 1 || p->window > p->chunk_size) return LZR_ERR_INVALID_ARG;
+  if (p->min_match < 3 || p->min_match > 255) return LZR_ERR_INVALID_ARG;
+  if (p->max_match < p->min_match || p->max_match > p->min_match + 255) return LZR_ERR_INVALID_ARG;
+  if (p->tie_break != LZR_TIE_LONGEST_THEN_NEAREST) return LZR_ERR_UNSUPPORTED;
+  return LZR_OK;
+}
+
+size_t lzr_num_chunks(size_t n_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK) return 0;
+  return (n_bytes + p->chunk_size - 1) / p->chunk_size;
+}
+
+size_t lzr_compress_bound(size_t n_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK) return 0;
+  return n_bytes;
+}
+
+size_t lzr_compress_workspace_bytes(size_t n_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK) return 0;
+  return ws_layout(n_bytes, p).total;
+}
+
+size_t lzr_scan_workspace_bytes(size_t n) { return scan_ws_bytes(n); }
+
+int lzr_last_launch_count(void) { return t_launches; }
+
+const char* lzr_status_str(int s) {
+  switch (s) {
+    case LZR_OK: return "LZR_OK";
+    case LZR_ERR_INVALID_ARG: return "LZR_ERR_INVALID_ARG";
+    case LZR_ERR_UNSUPPORTED: return "LZR_ERR_UNSUPPORTED";
+    case LZR_ERR_CAPACITY: return "LZR_ERR_CAPACITY";
+    case LZR_ERR_CUDA: return "LZR_ERR_CUDA";
+    case LZR_ERR_CORRUPT: return "LZR_ERR_CORRUPT";
+    default: return "LZR_ERR_UNKNOWN";
+  }
+}
+
+int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, uint32_t* d_sizes,
+                        void* d_workspace, size_t workspace_bytes, lzr_stream_t stream) {
+  t_launches = 0;
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  if (n_bytes == 0) return LZR_OK;
+  if (!d_in || !d_sizes || !d_workspace) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_in, 16) || !aligned(d_sizes, 4) || !aligned(d_workspace, 256))
+    return LZR_ERR_INVALID_ARG;
+  const WsLayout w = ws_layout(n_bytes, p);
+  if (workspace_bytes < w.total) return LZR_ERR_CAPACITY;
+  const size_t N = (n_bytes + p->chunk_size - 1) / p->chunk_size;
+  if (N > 0xFFFFFFFFull) return LZR_ERR_UNSUPPORTED;
+  DevInfo di;
+  if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
+  EncArgs a;
+  a.in = (const uint8_t*)d_in;
+  a.n_bytes = n_bytes;
+  a.N = (uint32_t)N;
+  a.C = p->chunk_size;
+  a.W = p->window;
+  a.m = p->min_match;
+  a.M = p->max_match;
+  a.kbytes = p->min_match < 4 ? p->min_match : 4;
+  a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
+  a.L = enc_layout(p->chunk_size);
+  if ((int)a.L.per_warp > di.smem_optin) return LZR_ERR_UNSUPPORTED;
+  uint8_t* ws = (uint8_t*)d_workspace;
+  a.slots = ws + w.slots_off;
+  a.sizes = d_sizes;
+  a.counter = (uint32_t*)(ws + w.ctrl_off);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (cudaMemsetAsync(ws + w.ctrl_off, 0, 256, s) != cudaSuccess) return LZR_ERR_CUDA;
+  if (launch_encode(a, di.sm_count, di.smem_optin, s, &t_launches) != cudaSuccess) return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_compress_compact(const void* d_in, size_t n_bytes, const lzr_params* p, void* d_out,
+                         size_t out_capacity, const uint32_t* d_sizes, uint64_t* d_offsets,
+                         uint64_t* d_total, void* d_workspace, size_t workspace_bytes,
+                         lzr_stream_t stream) {
+  t_launches = 0;
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n_bytes == 0) {
+    if (d_total && cudaMemsetAsync(d_total, 0, 8, s) != cudaSuccess) return LZR_ERR_CUDA;
+    return LZR_OK;
+  }
+  if (!d_in || !d_out || !d_sizes || !d_offsets || !d_workspace) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_in, 16) || !aligned(d_sizes, 4) || !aligned(d_offsets, 8) ||
+      !aligned(d_workspace, 256) || (d_total && !aligned(d_total, 8)))
+    return LZR_ERR_INVALID_ARG;
+  if (out_capacity < n_bytes) return LZR_ERR_CAPACITY;
+  const WsLayout w = ws_layout(n_bytes, p);
+  if (workspace_bytes < w.total) return LZR_ERR_CAPACITY;
+  DevInfo di;
+  if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
+  const size_t N = (n_bytes + p->chunk_size - 1) / p->chunk_size;
+  uint8_t* ws = (uint8_t*)d_workspace;
+  if (launch_scan(d_sizes, N, 0, d_offsets, d_total, ws + w.scan_off, s, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  if (launch_compact((const uint8_t*)d_in, n_bytes, p->chunk_size, ws + w.slots_off, d_sizes,
+                     d_offsets, (uint8_t*)d_out, di.sm_count, s, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_compress_chunks(const void* d_in, size_t n_bytes, const lzr_params* p, void* d_out,
+                        size_t out_capacity, uint32_t* d_sizes, uint64_t* d_offsets,
+                        uint64_t* d_total, void* d_workspace, size_t workspace_bytes,
+                        lzr_stream_t stream) {
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  if (n_bytes && out_capacity < n_bytes) return LZR_ERR_CAPACITY;
+  if (n_bytes && (!d_out || !d_offsets)) return LZR_ERR_INVALID_ARG;
+  st = lzr_compress_encode(d_in, n_bytes, p, d_sizes, d_workspace, workspace_bytes, stream);
+  if (st) return st;
+  const int l1 = t_launches;
+  st = lzr_compress_compact(d_in, n_bytes, p, d_out, out_capacity, d_sizes, d_offsets, d_total,
+                            d_workspace, workspace_bytes, stream);
+  t_launches += l1;
+  return st;
+}
+
+int lzr_scan_sizes(const uint32_t* d_sizes, size_t n, uint64_t base, uint64_t* d_offsets,
+                   uint64_t* d_total, void* d_workspace, size_t workspace_bytes,
+                   lzr_stream_t stream) {
+  t_launches = 0;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n == 0) {
+    if (d_total) {
+      // *d_total = base
+      if (cudaMemcpyAsync(d_total, &base, 8, cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return LZR_ERR_CUDA;
+      if (cudaStreamSynchronize(s) != cudaSuccess) return LZR_ERR_CUDA;
+    }
+    return LZR_OK;
+  }
+  if (!d_sizes || !d_offsets || !d_workspace) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_sizes, 4) || !aligned(d_offsets, 8) || !aligned(d_workspace, 256) ||
+      (d_total && !aligned(d_total, 8)))
+    return LZR_ERR_INVALID_ARG;
+  if (workspace_bytes < scan_ws_bytes(n)) return LZR_ERR_CAPACITY;
+  if (launch_scan(d_sizes, n, base, d_offsets, d_total, d_workspace, s, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_decompress_chunks(const void* d_comp, const uint32_t* d_sizes, const uint64_t* d_offsets,
+                          size_t n_bytes, const lzr_params* p, void* d_out, int32_t* d_error,
+                          lzr_stream_t stream) {
+  t_launches = 0;
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n_bytes && (!d_comp || !d_sizes || !d_offsets || !d_out)) return LZR_ERR_INVALID_ARG;
+  if (d_error && !aligned(d_error, 4)) return LZR_ERR_INVALID_ARG;
+  if (n_bytes && (!aligned(d_sizes, 4) || !aligned(d_offsets, 8))) return LZR_ERR_INVALID_ARG;
+  DevInfo di;
+  if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
+  if ((int)align_up(p->chunk_size + 16, 16) > di.smem_optin) return LZR_ERR_UNSUPPORTED;
+  if (launch_decode((const uint8_t*)d_comp, d_sizes, d_offsets, n_bytes, p->chunk_size,
+                    p->min_match, (uint8_t*)d_out, d_error, di.sm_count, di.smem_optin, s,
+                    &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+// ---- host-buffer end-to-end pipeline ---------------------------------------
+
+namespace {
+struct HostSet {
+  uint8_t *in, *out, *ws;
+  uint32_t* sizes;
+  uint64_t *offs, *total;
+  size_t ws_bytes;
+};
+
+size_t set_bytes(size_t batch, const lzr_params* p) {
+  const size_t C = p->chunk_size;
+  const size_t N = (batch + C - 1) / C;
+  return align_up_z(batch, 256) * 2 + align_up_z(4 * N, 256) + align_up_z(8 * N, 256) + 256 +
+         ws_layout(batch, p).total;
+}
+
+HostSet carve(uint8_t* base, size_t batch, const lzr_params* p) {
+  const size_t C = p->chunk_size;
+  const size_t N = (batch + C - 1) / C;
+  HostSet h;
+  size_t o = 0;
+  h.in = base + o; o += align_up_z(batch, 256);
+  h.out = base + o; o += align_up_z(batch, 256);
+  h.sizes = (uint32_t*)(base + o); o += align_up_z(4 * N, 256);
+  h.offs = (uint64_t*)(base + o); o += align_up_z(8 * N, 256);
+  h.total = (uint64_t*)(base + o); o += 256;
+  h.ws = base + o;
+  h.ws_bytes = ws_layout(batch, p).total;
+  return h;
+}
+}  // namespace
+
+size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
+  return 2 * align_up_z(set_bytes(batch_bytes, p), 256);
+}
+
+int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, void* h_out,
+                      size_t out_capacity, uint32_t* h_sizes, uint64_t* h_offsets,
+                      uint64_t* h_total, size_t batch_bytes, void* d_scratch,
+                      size_t scratch_bytes) {
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  const size_t C = p->chunk_size;
+  if (n_bytes == 0) {
+    if (h_total) *h_total = 0;
+    return LZR_OK;
+  }
+  if (!h_in || !h_out || !h_sizes || !h_offsets || !d_scratch) return LZR_ERR_INVALID_ARG;
+  if (out_capacity < n_bytes) return LZR_ERR_CAPACITY;
+  if (batch_bytes == 0) batch_bytes = align_up_z(n_bytes, C);
+  if (batch_bytes % C) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_scratch, 256)) return LZR_ERR_INVALID_ARG;
+  const size_t per = align_up_z(set_bytes(batch_bytes, p), 256);
+  if (scratch_bytes < 2 * per) return LZR_ERR_CAPACITY;
+  HostSet set[2] = {carve((uint8_t*)d_scratch, batch_bytes, p),
+                    carve((uint8_t*)d_scratch + per, batch_bytes, p)};
+  cudaStream_t s[2];
+  if (cudaStreamCreateWithFlags(&s[0], cudaStreamNonBlocking) != cudaSuccess) return LZR_ERR_CUDA;
+  if (cudaStreamCreateWithFlags(&s[1], cudaStreamNonBlocking) != cudaSuccess) {
+    cudaStreamDestroy(s[0]);
+    return LZR_ERR_CUDA;
+  }
+  const size_t nb = (n_bytes + batch_bytes - 1) / batch_bytes;
+  const size_t chunks_per_batch = batch_bytes / C;
+  uint64_t running = 0;
+  int rc = LZR_OK;
+  int launches = 0;
+  auto issue = [&](size_t b) -> int {
+    HostSet& h = set[b & 1];
+    const size_t lo = b * batch_bytes;
+    const size_t len = n_bytes - lo < batch_bytes ? n_bytes - lo : batch_bytes;
+    const size_t c0 = b * chunks_per_batch;
+    const size_t N = (len + C - 1) / C;
+    cudaStream_t ss = s[b & 1];
+    if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, ss) != cudaSuccess)
+      return LZR_ERR_CUDA;
+    int r = lzr_compress_chunks(h.in, len, p, h.out, batch_bytes, h.sizes, h.offs, h.total, h.ws,
+                                h.ws_bytes, (lzr_stream_t)ss);
+    if (r) return r;
+    launches += t_launches;
+    if (cudaMemcpyAsync(h_sizes + c0, h.sizes, 4 * N, cudaMemcpyDeviceToHost, ss) != cudaSuccess ||
+        cudaMemcpyAsync(h_offsets + c0, h.offs, 8 * N, cudaMemcpyDeviceToHost, ss) != cudaSuccess)
+      return LZR_ERR_CUDA;
+    return LZR_OK;
+  };
+  auto finish = [&](size_t b) -> int {
+    HostSet& h = set[b & 1];
+    cudaStream_t ss = s[b & 1];
+    if (cudaStreamSynchronize(ss) != cudaSuccess) return LZR_ERR_CUDA;
+    const size_t lo = b * batch_bytes;
+    const size_t len = n_bytes - lo < batch_bytes ? n_bytes - lo : batch_bytes;
+    const size_t c0 = b * chunks_per_batch;
+    const size_t N = (len + C - 1) / C;
+    uint64_t tb = 0;  // batch total = sum of its sizes (already on the host)
+    for (size_t i = 0; i < N; ++i) {
+      h_offsets[c0 + i] += running;
+      tb += h_sizes[c0 + i];
+    }
+    if (tb && cudaMemcpyAsync((uint8_t*)h_out + running, h.out, tb, cudaMemcpyDeviceToHost, ss) != cudaSuccess)
+      return LZR_ERR_CUDA;
+    running += tb;
+    return LZR_OK;
+  };
+  for (size_t b = 0; b < nb && rc == LZR_OK; ++b) {
+    rc = issue(b);
+    if (rc == LZR_OK && b >= 1) rc = finish(b - 1);
+  }
+  if (rc == LZR_OK) rc = finish(nb - 1);
+  if (cudaStreamSynchronize(s[0]) != cudaSuccess || cudaStreamSynchronize(s[1]) != cudaSuccess)
+    rc = rc ? rc : LZR_ERR_CUDA;
+  cudaStreamDestroy(s[0]);
+  cudaStreamDestroy(s[1]);
+  if (h_total) *h_total = running;
+  t_launches = launches;
+  return rc;
+}
+
+}  // extern "C"

@@ -1,0 +1,131 @@
+// lzr_internal.cuh -- device helpers and launch plumbing shared by the sm_100a
+// kernels of liblzr.so (encode, scan/compact, decode).  Part of the CUDA path
+// only; the oracle (oracle/) shares nothing with it.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/lzr.h"
+
+namespace lzr {
+
+constexpr uint32_t kFull = 0xFFFFFFFFu;
+
+__host__ __device__ constexpr uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
+__host__ __device__ constexpr size_t align_up_z(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// Unaligned little-endian 32-bit load from a shared-memory byte buffer whose
+// base is 16-byte aligned: two aligned LDS.32 + one funnel shift.
+__device__ __forceinline__ uint32_t ld32u(const uint8_t* base, uint32_t p) {
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(base);
+  uint32_t a = w[p >> 2];
+  uint32_t b = w[(p >> 2) + 1];
+  return __funnelshift_r(a, b, (p & 3u) << 3);
+}
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// ---- mbarrier + 1-D bulk TMA (cp.async.bulk) ---------------------------------
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_bulk_g2s(void* smem_dst, const void* gmem_src, uint32_t bytes,
+                                             uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(smem_dst)),
+      "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+  }
+}
+
+// ---- encode kernel shared-memory layout (one region per warp = per chunk) ---
+struct EncLayout {
+  uint32_t off_sorted, off_slot, off_bm, off_mbar, per_warp, hbits, bm_words;
+};
+
+__host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
+  uint32_t hb = 0;
+  while ((2u << hb) <= C && hb < 12) ++hb;  // largest power of two <= C, capped at 4096
+  return hb;
+}
+
+__host__ __device__ inline EncLayout enc_layout(uint32_t C) {
+  EncLayout L;
+  L.hbits = enc_hash_bits(C);
+  uint32_t B = 1u << L.hbits;
+  uint32_t o = align_up(C + 16, 16);  // chunk bytes + zero pad for unaligned word loads
+  L.off_sorted = o;
+  o = align_up(o + 2 * C, 16);  // u16 positions grouped by hash bucket, ascending
+  L.off_slot = o;
+  o = align_up(o + 2 * (C > B ? C : B), 16);  // u16 slot of each position (histogram before)
+  L.off_bm = o;
+  L.bm_words = C / 32 + 2;
+  o = align_up(o + 4 * L.bm_words, 16);  // candidate bitmap (1 bit per position)
+  L.off_mbar = o;
+  o += 16;
+  L.per_warp = align_up(o, 128);
+  return L;
+}
+
+struct EncArgs {
+  const uint8_t* in;
+  size_t n_bytes;
+  uint32_t N;  // chunks (fits: N <= 2^32 - 1 checked on host)
+  uint32_t C, W, m, M;
+  uint32_t kbytes, kmask;  // candidate key = first min(m,4) bytes
+  EncLayout L;
+  uint8_t* slots;  // workspace: chunk i stream at slots + i*C
+  uint32_t* sizes;
+  uint32_t* counter;  // work distribution, zeroed before launch
+};
+
+// ---- workspace layout ---------------------------------------------------------
+struct WsLayout {
+  size_t ctrl_off, slots_off, scan_off, total;
+};
+size_t scan_ws_bytes(size_t n);
+WsLayout ws_layout(size_t n_bytes, const lzr_params* p);
+
+// launches (defined in the .cu files); return cudaError_t of the launch
+cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches);
+cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, uint64_t* offsets,
+                        uint64_t* total, void* ws, cudaStream_t s, int* launches);
+cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const uint8_t* slots,
+                           const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,
+                           int sm_count, cudaStream_t s, int* launches);
+cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,
+                          size_t n_bytes, uint32_t C, uint32_t m, uint8_t* out, int32_t* err,
+                          int sm_count, int smem_optin, cudaStream_t s, int* launches);
+
+}  // namespace lzr

@@ -1,0 +1,128 @@
+"""Multi-GPU sharding of chunk batches.
+
+Chunks are independent (§3.2(1) "there is no data dependency between
+chunks"), so rank r of R compresses a contiguous chunk range on its own GPU.
+The only exchange step is the one the global layout needs: every rank
+all-gathers the per-chunk uint32 compressed sizes (NCCL over NVLink /
+NVSwitch) and derives the global offsets with the device scan of liblzr
+(``lzr_scan_sizes``).  Compressed bytes never leave their rank.
+
+Shards are padded to ceil(N/R) chunks with zero sizes, so the gathered array
+is [R, ceil(N/R)] and its exclusive scan directly gives every real chunk's
+global offset (padding contributes 0) -- no reshuffle on the data path.
+
+The compress / scan / collective steps are taken from an ``ops`` object; the
+default is the CUDA path (liblzr) with ``torch.distributed`` collectives.
+Tests substitute a CPU implementation to exercise the host-side shard and
+offset logic over a gloo group; there is no CPU fallback in the product path.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as dist
+
+from . import Params, Workspace, compress, num_chunks, scan_sizes
+
+
+def shard_range(n_chunks: int, world: int, rank: int) -> tuple[int, int]:
+    """Contiguous chunk range [lo, hi) of `rank`; the remainder goes to the first ranks."""
+    base, rem = divmod(n_chunks, world)
+    lo = rank * base + min(rank, rem)
+    return lo, lo + base + (1 if rank < rem else 0)
+
+
+def max_shard(n_chunks: int, world: int) -> int:
+    return -(-n_chunks // world)
+
+
+class CudaOps:
+    """The product path: liblzr kernels + torch.distributed collectives."""
+
+    def __init__(self, p: Params, n_local: int, device):
+        self.p = p
+        self.ws = Workspace(n_local, p, device)
+
+    def bind_sizes(self, sizes_pad):
+        # the encoder writes the per-chunk sizes straight into the padded
+        # all-gather input (no copy on the data path)
+        self.ws.sizes = sizes_pad
+
+    def compress(self, x):
+        out, sizes, offsets, total = compress(x, self.p, ws=self.ws)
+        return out, sizes, total
+
+    def scan(self, sizes_all, offsets, total):
+        scan_sizes(sizes_all, 0, offsets=offsets, total=total)
+
+    def all_gather(self, out, inp, group):
+        dist.all_gather_into_tensor(out, inp, group=group)
+
+
+@dataclass
+class ShardResult:
+    out: torch.Tensor            # local compacted streams (first local_total bytes valid)
+    local_sizes: torch.Tensor    # [N_r] int32
+    local_total: torch.Tensor    # [1] int64
+    sizes_all: torch.Tensor      # [R * maxN] int32, zero-padded per rank
+    offsets_all: torch.Tensor    # [R * maxN] int64 global exclusive offsets
+    global_total: torch.Tensor   # [1] int64
+    lo: int
+    hi: int
+    max_n: int
+
+    def global_offsets(self) -> torch.Tensor:
+        """Global offsets of this rank's chunks (view)."""
+        r = self.lo_rank
+        return self.offsets_all[r * self.max_n: r * self.max_n + (self.hi - self.lo)]
+
+
+class ShardedCompressor:
+    """compress_sharded with persistent buffers (one instance per rank)."""
+
+    def __init__(self, n_bytes_global: int, p: Params, group=None, device=None, ops=None):
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.p = p
+        self.N = num_chunks(n_bytes_global, p)
+        self.n_global = n_bytes_global
+        self.lo, self.hi = shard_range(self.N, self.world, self.rank)
+        self.max_n = max(1, max_shard(self.N, self.world))
+        self.byte_lo = self.lo * p.chunk_size
+        self.byte_hi = min(n_bytes_global, self.hi * p.chunk_size)
+        self.n_local = self.byte_hi - self.byte_lo
+        dev = torch.device(device) if device is not None else None
+        self.ops = ops if ops is not None else CudaOps(p, self.n_local, dev)
+        kw = dict(device=dev) if dev is not None else {}
+        self.sizes_pad = torch.zeros(self.max_n, dtype=torch.int32, **kw)
+        self.sizes_all = torch.zeros(self.world * self.max_n, dtype=torch.int32, **kw)
+        self.offsets_all = torch.zeros(self.world * self.max_n, dtype=torch.int64, **kw)
+        self.global_total = torch.zeros(1, dtype=torch.int64, **kw)
+        if hasattr(self.ops, "bind_sizes"):
+            self.ops.bind_sizes(self.sizes_pad)
+
+    def __call__(self, x_local) -> ShardResult:
+        """x_local: this rank's bytes [byte_lo, byte_hi) of the global stream."""
+        assert x_local.numel() == self.n_local
+        nl = self.hi - self.lo
+        if nl:
+            out, sizes, total = self.ops.compress(x_local)
+            if sizes.data_ptr() != self.sizes_pad.data_ptr():
+                self.sizes_pad[:nl].copy_(sizes[:nl])
+        else:
+            out = x_local.new_empty(0)
+            sizes = self.sizes_pad[:0]
+            total = torch.zeros(1, dtype=torch.int64, device=self.sizes_pad.device)
+        self.ops.all_gather(self.sizes_all, self.sizes_pad, self.group)
+        self.ops.scan(self.sizes_all, self.offsets_all, self.global_total)
+        res = ShardResult(out, sizes[:nl], total, self.sizes_all, self.offsets_all,
+                          self.global_total, self.lo, self.hi, self.max_n)
+        res.lo_rank = self.rank
+        return res
+
+
+def compress_sharded(x_local, p: Params, n_bytes_global: int, group=None):
+    """One-shot convenience wrapper (allocates buffers every call)."""
+    return ShardedCompressor(n_bytes_global, p, group, x_local.device)(x_local)

@@ -1,0 +1,219 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+byte for byte (0-byte tolerance on output bytes, sizes and offsets; integer
+work, so bit-exact is the bar -- DESIGN.md §Parity).
+
+Sizes span several warps/CTAs and ragged tails; the full-size config-2 case
+checks a deterministic chunk sample against the oracle plus a full GPU round
+trip, in the launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+pytestmark = pytest.mark.gpu
+
+import synth  # noqa: E402
+
+
+@pytest.fixture(scope="module")
+def lzr():
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    import __graft_entry__
+
+    __graft_entry__.build()
+    import paper_conf_pact_map17_b200 as m
+
+    return m
+
+
+def _ref_params(ref, p):
+    return ref.Params(chunk_size=p.chunk_size, window=p.window, min_match=p.min_match,
+                      max_match=p.max_match)
+
+
+def _gpu_compress(lzr, x: np.ndarray, p):
+    xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
+    out, sizes, offs, total = lzr.compress(xd, p)
+    torch.cuda.synchronize()
+    tot = int(total.item())
+    return (xd, out, sizes, offs, tot,
+            out[:tot].cpu().numpy(), sizes.cpu().numpy().view(np.uint32),
+            offs.cpu().numpy().view(np.uint64))
+
+
+def _check_full(lzr, ref, x: np.ndarray, p, roundtrip=True):
+    xd, out, sizes, offs, tot, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, p)
+    r_out, r_sizes, r_offs, r_tot = ref.compress(x, _ref_params(ref, p))
+    assert tot == r_tot
+    assert np.array_equal(g_sizes, r_sizes)
+    assert np.array_equal(g_offs, r_offs)
+    if not np.array_equal(g_out, r_out):
+        bad = int(np.argmax(g_out != r_out))
+        ci = int(np.searchsorted(r_offs, bad, side="right") - 1)
+        raise AssertionError(f"first differing byte {bad} in chunk {ci}")
+    if roundtrip:
+        y, err = lzr.decompress(out, sizes, offs, x.size, p)
+        torch.cuda.synchronize()
+        assert int(err.item()) == 0
+        assert torch.equal(y, xd)
+    return g_out, g_sizes, g_offs
+
+
+def test_config1_mix_bitexact(lzr, ref):
+    x = synth.fill_host(1 << 20, 4096, "mix")
+    _check_full(lzr, ref, x, lzr.Params())
+
+
+@pytest.mark.parametrize("cls", ["text", "random", "zeroruns", "cr2"])
+def test_classes_bitexact(lzr, ref, cls):
+    x = synth.fill_host(1 << 20, 4096, cls, seed=11)
+    _check_full(lzr, ref, x, lzr.Params())
+
+
+def _adversarial():
+    rng = np.random.default_rng(5)
+    yield "zeros", np.zeros(4096 * 9, np.uint8)
+    yield "ones_ragged", np.full(4096 * 3 + 5, 0xFF, np.uint8)
+    yield "random_ragged", rng.integers(0, 256, 4096 * 5 + 1234, dtype=np.uint8)
+    for q in [1, 2, 3, 4, 5, 7, 8, 16, 31, 32, 33, 63, 64, 200]:
+        base = rng.integers(0, 256, q, dtype=np.uint8)
+        yield f"period{q}", np.tile(base, 4096 * 2 // q + 2)[: 4096 * 2 + 77]
+    yield "binary", rng.integers(0, 2, 4096 * 6, dtype=np.uint8)
+    yield "quaternary", rng.integers(0, 4, 4096 * 6, dtype=np.uint8) + 0x61
+    yield "runs", np.repeat(rng.integers(0, 3, 4000, dtype=np.uint8), rng.integers(1, 40, 4000))[: 4096 * 8]
+    yield "tiny1", np.array([7], np.uint8)
+    yield "tiny5", np.frombuffer(b"aaaaa", np.uint8).copy()
+
+
+@pytest.mark.parametrize("name,x", list(_adversarial()), ids=lambda v: v if isinstance(v, str) else "")
+def test_adversarial_bitexact(lzr, ref, name, x):
+    _check_full(lzr, ref, x, lzr.Params())
+
+
+@pytest.mark.parametrize("C,W,m,M", [
+    (4096, 4096, 3, 258), (4096, 4096, 5, 40), (4096, 4096, 4, 4), (4096, 4096, 4, 5),
+    (4096, 1000, 4, 259), (4096, 1, 4, 259), (4096, 2, 3, 100), (4096, 33, 6, 261),
+    (16, 16, 3, 258), (16, 5, 4, 259), (48, 48, 4, 259), (528, 300, 4, 20),
+    (8192, 8192, 4, 259), (16384, 16384, 4, 259), (32768, 32768, 4, 259),
+])
+def test_param_grid_bitexact(lzr, ref, C, W, m, M):
+    p = lzr.Params(chunk_size=C, window=W, min_match=m, max_match=M)
+    n = max(C * 3 + C // 3 + 1, 3000)
+    x = synth.fill_host(n, C, "mix", seed=C + W + m + M)
+    _check_full(lzr, ref, x, p)
+
+
+@pytest.mark.parametrize("nchunks", [1, 2, 31, 32, 33, 147, 148, 149, 11 * 148 - 1, 11 * 148 + 1])
+def test_batch_edges(lzr, ref, nchunks):
+    x = synth.fill_host(nchunks * 4096, 4096, "mix", seed=nchunks)
+    _check_full(lzr, ref, x, lzr.Params(), roundtrip=True)
+
+
+def test_golden_through_gpu(lzr, ref):
+    import json, os
+    path = os.path.join(os.path.dirname(__file__), "golden", "appendix_a.jsonl")
+    for line in open(path):
+        c = json.loads(line)
+        pp = c["params"]
+        p = lzr.Params(chunk_size=pp["chunk_size"], window=pp["window"], min_match=pp["min_match"],
+                       max_match=pp["max_match"])
+        if "input_ascii" in c:
+            x = np.frombuffer(c["input_ascii"].encode(), np.uint8).copy()
+        else:
+            x = np.full(c["input_fill"][1], c["input_fill"][0], np.uint8)
+        _, _, _, _, tot, g_out, g_sizes, _ = _gpu_compress(lzr, x, p)
+        assert tot == c["size"] and g_out.tobytes().hex() == c["expected_hex"], c["id"]
+
+
+def test_config2_full_size_sampled(lzr, ref):
+    """256 MiB mix at the bench's launch configuration: deterministic sample
+    (every 256th chunk + first/last 64) vs the oracle, full round trip."""
+    n = 256 << 20
+    p = lzr.Params()
+    xd = torch.empty(n, dtype=torch.uint8, device="cuda")
+    synth.fill_device(xd, 4096, "mix")
+    x = xd.cpu().numpy()
+    assert np.array_equal(x[: 1 << 20], synth.fill_host(1 << 20, 4096, "mix"))  # host == device gen
+    out, sizes, offs, total = lzr.compress(xd, p)
+    torch.cuda.synchronize()
+    N = n // 4096
+    idx = sorted(set(range(0, N, 256)) | set(range(64)) | set(range(N - 64, N)))
+    g_sizes = sizes.cpu().numpy().view(np.uint32)
+    g_offs = offs.cpu().numpy().view(np.uint64)
+    g_out = out.cpu().numpy()
+    r_streams, r_sizes = ref.compress_sampled(x, _ref_params(ref, p), idx)
+    for k, i in enumerate(idx):
+        assert g_sizes[i] == r_sizes[k], i
+        assert g_out[g_offs[i]: g_offs[i] + g_sizes[i]].tobytes() == r_streams[k], i
+    assert g_offs[0] == 0 and np.array_equal(g_offs[1:], np.cumsum(g_sizes[:-1], dtype=np.uint64))
+    assert int(total.item()) == int(g_sizes.sum(dtype=np.uint64))
+    y, err = lzr.decompress(out, sizes, offs, n, p)
+    torch.cuda.synchronize()
+    assert int(err.item()) == 0 and torch.equal(y, xd)
+
+
+def test_cross_decode_with_oracle(lzr, ref):
+    x = synth.fill_host(3 << 20, 4096, "cr2", seed=99)
+    g_out, g_sizes, g_offs = _check_full(lzr, ref, x, lzr.Params(), roundtrip=False)
+    st, bad, y = ref.decompress(g_out, g_sizes, g_offs, x.size, ref.Params())
+    assert st == 0 and np.array_equal(y, x)
+
+
+def test_gpu_decoder_matches_oracle_on_corruption(lzr, ref):
+    x = synth.fill_host(64 * 4096, 4096, "text", seed=3)
+    p = lzr.Params()
+    xd, out, sizes, offs, tot, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, p)
+    rng = np.random.default_rng(1)
+    for trial in range(40):
+        bad = g_out.copy()
+        bs = g_sizes.copy()
+        kind = trial % 3
+        ci = int(rng.integers(0, 64))
+        if g_sizes[ci] == 4096:
+            continue
+        if kind == 0:  # flip a random byte inside chunk ci
+            pos = int(g_offs[ci] + rng.integers(0, g_sizes[ci]))
+            bad[pos] ^= np.uint8(1 << int(rng.integers(0, 8)))
+        elif kind == 1:  # truncate chunk ci by one byte
+            bs[ci] -= 1
+        else:  # claim one more byte
+            bs[ci] += 1 if bs[ci] + 1 < 4096 else 0
+        st, r_bad, _ = ref.decompress(bad, bs, g_offs, x.size, ref.Params())
+        d_bad = torch.from_numpy(bad).cuda()
+        d_bs = torch.from_numpy(bs.view(np.int32)).cuda()
+        _, err = lzr.decompress(d_bad, d_bs, offs, x.size, p)
+        torch.cuda.synchronize()
+        assert int(err.item()) == r_bad, (trial, kind, ci)
+
+
+def test_scan_sizes_large(lzr):
+    rng = np.random.default_rng(2)
+    for n in [1, 7, 2048, 2049, 100003, 5_000_000]:
+        s = rng.integers(0, 4097, n, dtype=np.uint32)
+        d = torch.from_numpy(s.view(np.int32)).cuda()
+        offs, tot = lzr.scan_sizes(d, base=12345)
+        torch.cuda.synchronize()
+        exp = np.concatenate([[0], np.cumsum(s[:-1], dtype=np.uint64)]) + np.uint64(12345)
+        assert np.array_equal(offs.cpu().numpy().view(np.uint64), exp)
+        assert int(tot.item()) == 12345 + int(s.sum(dtype=np.uint64))
+
+
+def test_compress_host_pipeline(lzr, ref):
+    n = (8 << 20) + 4096 * 3 + 100
+    x = synth.fill_host(n, 4096, "mix", seed=21)
+    h = torch.from_numpy(x).pin_memory()
+    for batch in [0, 1 << 20, 3 * 4096 * 128]:
+        h_out, h_sizes, h_offs, tot = lzr.compress_host(h, lzr.Params(), batch_bytes=batch)
+        xd, out, sizes, offs, dtot, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, lzr.Params())
+        assert tot == dtot
+        assert np.array_equal(h_sizes.numpy().view(np.uint32), g_sizes)
+        assert np.array_equal(h_offs.numpy().view(np.uint64), g_offs)
+        assert np.array_equal(h_out[:tot].numpy(), g_out)
+
+
+def test_empty_input(lzr):
+    xd = torch.empty(0, dtype=torch.uint8, device="cuda")
+    out, sizes, offs, total = lzr.compress(xd, lzr.Params())
+    torch.cuda.synchronize()
+    assert sizes.numel() == 0 and int(total.item()) == 0
