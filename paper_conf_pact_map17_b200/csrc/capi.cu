@@ -129,7 +129,9 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.kbytes = p->min_match < 4 ? p->min_match : 4;
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
   a.L = enc_layout(p->chunk_size);
-  if ((int)a.L.per_warp > di.smem_optin) return LZR_ERR_UNSUPPORTED;
+  // positions are 15-bit in the index (bit 15 marks bucket starts) and one
+  // chunk's index must fit one CTA's shared memory
+  if (p->chunk_size > 32768 || (int)a.L.per_warp > di.smem_optin) return LZR_ERR_UNSUPPORTED;
   uint8_t* ws = (uint8_t*)d_workspace;
   a.slots = ws + w.slots_off;
   a.sizes = d_sizes;

@@ -4,24 +4,30 @@
 // threads for each chunk. Each stage performs its own LZ compression algorithm
 // with its own history buffer and look-ahead buffer."):
 //   a2  stage the chunk (= its whole history window, R2) into shared memory with
-//       a 1-D bulk TMA copy (cp.async.bulk + mbarrier);
-//   a3  longest-match search.  Exact candidates are the earlier positions with
-//       the same first k = min(m,4) bytes (any match of length >= m >= k starts
-//       with them).  The warp counting-sorts positions by a hash of that key
-//       into buckets that stay in ascending position order, so the candidates of
-//       p are a contiguous run of slots below p's own slot, nearest first.  The
-//       32 lanes evaluate 32 candidates at a time; each candidate's capped
-//       common-prefix length is packed as (len << 16 | 0xFFFF - (d - 1)) and
-//       reduced with REDUX.MAX, which selects "longest, then nearest" (R6, R7).
-//       A candidate beyond the best length so far must also match the byte at
-//       that length (a necessary condition for being strictly longer), so most
-//       farther candidates cost one compare.  Search stops at the cap (exact:
-//       nothing beats the cap) or when the bucket / window is exhausted.
-//   a4  greedy selection (R8): the warp walks p = 0 .. n-1.  A 1-bit-per-position
-//       "has a same-key candidate inside the window" bitmap lets it emit runs of
-//       up to 32 literals per step (ballot-free: one funnel shift of the bitmap).
-//   a5  flag-byte LZSS encoding (R1) straight into the chunk's workspace slot,
-//       raw fallback when the stream would not be shorter than the chunk (R9).
+//       a 1-D bulk TMA copy (cp.async.bulk + mbarrier).
+//   a3  index: exact candidates of p are the earlier positions with the same
+//       first k = min(m,4) bytes (a match of length >= m >= k starts with them).
+//       The warp counting-sorts positions by a hash of that key into buckets
+//       kept in ascending position order (stable scatter, MATCH.ANY ranks); bit
+//       15 of an entry marks the first entry of its bucket.  A per-position bit
+//       says whether a same-key position exists inside the window, and a
+//       "byte changes here" bitmap gives run lengths in O(1) for the run
+//       shortcut below.
+//   a3  longest match at a token start p: the 32 lanes take the 32 nearest
+//       candidates (slots below p's own), compute the capped common-prefix
+//       length with 16-byte compares (or, when both sides start inside runs of
+//       the same byte, straight from the two run lengths), pack
+//       (len << 16 | 0xFFFF - (d-1)) and reduce with REDUX.MAX = "longest, then
+//       nearest" (R6, R7).  A farther candidate must also match the byte at the
+//       best length so far to be strictly longer, so most cost one compare.
+//       Stop at the cap (exact: nothing beats it) or when bucket/window end.
+//   a4  greedy walk (R8): literal runs advance up to 32 positions per step via
+//       the candidate bitmap; the walk only records token starts, match bits,
+//       (d-1) and (l-m) in place and keeps the running stream size, so a chunk
+//       whose stream reaches n bytes is stored raw (R9) without encoding.
+//   a5  encode (R1) in parallel over positions: token index and match count by
+//       ballot/popc prefix sums give every token's output byte position; the
+//       stream is assembled in shared memory and written with 16-byte stores.
 // The serial result is reproduced exactly: the best match at p depends only on
 // (chunk bytes, p, W, m, M), not on the parse.
 #include "lzr_internal.cuh"
@@ -31,135 +37,136 @@ namespace lzr {
 namespace {
 
 constexpr int kMaxWarps = 16;
+constexpr uint16_t kFirst = 0x8000;  // first entry of its bucket
+constexpr uint16_t kPos = 0x7FFF;
+constexpr uint32_t kMaxRuns = 32;  // runs of one byte value of length >= k, per chunk
 
 __device__ __forceinline__ uint32_t khash(uint32_t key, uint32_t hbits) {
   return (key * 0x9E3779B1u) >> (32 - hbits);
 }
 
-// Capped common-prefix length of data[a..] and data[b..] (a > b allowed to
-// overlap: compares original bytes, = byte-serial copy semantics, R5).
-__device__ __forceinline__ uint32_t lcp_words(const uint8_t* d, uint32_t a, uint32_t b,
-                                              uint32_t maxlen) {
+// Common-prefix length of data[a..] and data[b..], capped at maxlen; 16 bytes
+// per step (5 aligned words per side + funnel shifts).  Overlap (a > b) is
+// allowed: original bytes are compared (= byte-serial copy semantics, R5).
+__device__ __forceinline__ uint32_t lcp16(const uint8_t* d, uint32_t a, uint32_t b,
+                                          uint32_t maxlen) {
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(d);
+  const uint32_t sa = (a & 3u) << 3, sb = (b & 3u) << 3;
+  uint32_t ia = a >> 2, ib = b >> 2;
+  uint32_t a0 = w[ia], b0 = w[ib];
   uint32_t l = 0;
   while (l < maxlen) {
-    uint32_t x = ld32u(d, a + l) ^ ld32u(d, b + l);
-    if (x) {
-      l += (uint32_t)(__ffs(x) - 1) >> 3;
+    const uint32_t a1 = w[ia + 1], a2 = w[ia + 2], a3 = w[ia + 3], a4 = w[ia + 4];
+    const uint32_t b1 = w[ib + 1], b2 = w[ib + 2], b3 = w[ib + 3], b4 = w[ib + 4];
+    const uint32_t x0 = __funnelshift_r(a0, a1, sa) ^ __funnelshift_r(b0, b1, sb);
+    const uint32_t x1 = __funnelshift_r(a1, a2, sa) ^ __funnelshift_r(b1, b2, sb);
+    const uint32_t x2 = __funnelshift_r(a2, a3, sa) ^ __funnelshift_r(b2, b3, sb);
+    const uint32_t x3 = __funnelshift_r(a3, a4, sa) ^ __funnelshift_r(b3, b4, sb);
+    if (x0 | x1 | x2 | x3) {
+      uint32_t k, x;
+      if (x0) { k = 0; x = x0; }
+      else if (x1) { k = 4; x = x1; }
+      else if (x2) { k = 8; x = x2; }
+      else { k = 12; x = x3; }
+      l += k + ((uint32_t)(__ffs(x) - 1) >> 3);
       return l < maxlen ? l : maxlen;
     }
-    l += 4;
+    l += 16;
+    ia += 4;
+    ib += 4;
+    a0 = a4;
+    b0 = b4;
   }
   return maxlen;
 }
 
-struct EncState {
-  uint32_t opos, fpos, cnt, fbits;
+// min(run length of the byte at p, lim): distance to the next set bit of the
+// change bitmap cb (bit i = x[i] != x[i-1]; set for i >= n).
+__device__ __forceinline__ uint32_t run_len(const uint32_t* cb, uint32_t p, uint32_t lim) {
+  uint32_t i = p + 1;
+  uint32_t wi = i >> 5;
+  uint32_t bits = cb[wi] >> (i & 31u);
+  uint32_t base = i;
+  while (bits == 0) {
+    ++wi;
+    base = wi << 5;
+    if (base - p >= lim) return lim;
+    bits = cb[wi];
+  }
+  const uint32_t r = base + (uint32_t)(__ffs(bits) - 1) - p;
+  return r < lim ? r : lim;
+}
+
+struct Smem {
+  uint8_t* data;
+  uint16_t* sorted;  // entries: position | kFirst; later: the output stream staging
+  uint16_t* slot;    // histogram/cursors during the sort; slot of each position;
+                     // after the walk: (d-1) at a match start, (l-m) right after it
+  uint32_t* cand;    // 1: a same-key position exists inside the window
+  uint32_t* cb;      // 1: byte differs from the previous one (run boundaries)
+  uint32_t* tb;      // 1: token starts here
+  uint32_t* mb;      // 1: the token here is a match
+  uint8_t* flags;    // flag byte of each group of 8 tokens
+  uint32_t* runs;    // (end << 16) | start of every run of >= k equal bytes (first kMaxRuns)
 };
 
-// Emit L (1..32) literal tokens x[p..p+L) (R1: literal = 1 byte, flag bit 0).
-__device__ __forceinline__ void emit_literals(uint8_t* out, const uint8_t* data, uint32_t p,
-                                              uint32_t L, uint32_t n, EncState& e,
-                                              uint32_t lane) {
-  const uint32_t c0 = e.cnt;
-  if (lane < L) {
-    uint32_t t = c0 + lane;
-    uint32_t nf = (c0 == 0) ? (lane >> 3) + 1 : (t >> 3);  // flag bytes opened up to this token
-    uint32_t pos = e.opos + lane + nf;
-    if (pos < n) out[pos] = data[p + lane];
-    // a group opened and completed inside this run holds only literals: flag 0
-    if ((t & 7u) == 0 && lane + 7 < L && pos - 1 < n) out[pos - 1] = 0;
-  }
-  // the group open before this run is completed inside it: its flag byte is final
-  if (c0 != 0 && c0 + L >= 8 && lane == 0 && e.fpos < n) out[e.fpos] = (uint8_t)e.fbits;
-  const uint32_t nf_tot = (c0 == 0) ? ((L - 1) >> 3) + 1 : ((c0 + L - 1) >> 3);
-  const uint32_t cend = (c0 + L) & 7u;
-  if (!(c0 != 0 && c0 + L < 8) && cend != 0) {
-    // a new group opened inside this run stays open
-    uint32_t ts = (c0 + L - 1) & ~7u;
-    uint32_t is = ts - c0;
-    uint32_t nfs = (c0 == 0) ? (is >> 3) + 1 : (ts >> 3);
-    e.fpos = e.opos + is + nfs - 1;
-    e.fbits = 0;
-  }
-  e.opos += L + nf_tot;
-  e.cnt = cend;
-}
-
-// Emit one match token (R1: 3 bytes (d-1) u16 LE, (l-m) u8; flag bit 1).
-__device__ __forceinline__ void emit_match(uint8_t* out, uint32_t d, uint32_t l, uint32_t m,
-                                           uint32_t n, EncState& e, uint32_t lane) {
-  if (e.cnt == 0) {
-    e.fpos = e.opos;
-    e.opos += 1;
-    e.fbits = 0;
-  }
-  if (lane == 0) {
-    uint32_t o = e.opos;
-    if (o < n) out[o] = (uint8_t)((d - 1) & 0xFF);
-    if (o + 1 < n) out[o + 1] = (uint8_t)((d - 1) >> 8);
-    if (o + 2 < n) out[o + 2] = (uint8_t)(l - m);
-  }
-  e.fbits |= 1u << e.cnt;
-  e.opos += 3;
-  e.cnt += 1;
-  if (e.cnt == 8) {
-    if (lane == 0 && e.fpos < n) out[e.fpos] = (uint8_t)e.fbits;
-    e.cnt = 0;
-  }
-}
-
-// Longest, then nearest, capped match at p (a3).  Returns the packed key
-// (len << 16) | (0xFFFF - (d-1)), or 0 when no candidate reaches m.
-__device__ __forceinline__ uint32_t best_match(const uint8_t* data, const uint16_t* sorted,
-                                               const uint16_t* slot, uint32_t p, uint32_t n,
-                                               const EncArgs& a, uint32_t lane) {
-  const uint32_t kp = ld32u(data, p) & a.kmask;
-  const uint32_t hp = khash(kp, a.L.hbits);
-  const uint32_t cap = min(a.M, n - p);  // p < n - m + 1  =>  cap >= m >= k
-  uint32_t best = 0, blen = 0;
-  for (int sb = (int)slot[p] - 1; sb >= 0; sb -= 32) {
-    const int s = sb - (int)lane;
-    uint32_t q = 0;
-    bool stop = true, cand = false;
-    if (s >= 0) {
-      q = sorted[s];
-      const uint32_t kq = ld32u(data, q) & a.kmask;
-      const bool in_window = p - q <= a.W;
-      stop = !in_window || (kq != kp && khash(kq, a.L.hbits) != hp);
-      cand = !stop && kq == kp;
-    }
-    const uint32_t stopmask = __ballot_sync(kFull, stop);
-    const uint32_t first_stop = stopmask ? (uint32_t)(__ffs(stopmask) - 1) : 32u;
-    uint32_t pk = 0;
-    if (cand && lane < first_stop) {
-      // strictly longer than blen requires a match at offset blen (blen < cap here)
-      if (blen == 0 || data[q + blen] == data[p + blen]) {
-        const uint32_t l = a.kbytes + lcp_words(data, p + a.kbytes, q + a.kbytes, cap - a.kbytes);
-        if (l >= a.m) pk = (l << 16) | (0xFFFFu - (p - q - 1));
-      }
-    }
-    best = max(best, __reduce_max_sync(kFull, pk));
-    blen = best >> 16;
-    if (blen >= cap || first_stop < 32) break;
-  }
-  return best;
-}
-
-// Build the per-chunk candidate structure (sorted buckets, slots, bitmap).
-__device__ __forceinline__ void build_index(const uint8_t* data, uint16_t* sorted, uint16_t* slot,
-                                            uint32_t* bm, uint32_t n, uint32_t P, const EncArgs& a,
-                                            uint32_t lane) {
+// ---- a3: index ----------------------------------------------------------------
+// Returns true when the chunk is certainly stored raw (R9) and the index was not
+// built.  Sound bound: a match of length l at p makes positions p..p+l-k
+// (k = key bytes) positions with a same-key earlier occurrence, disjoint across
+// matches; with X = sum(l - 3) and T tokens, S = n - X + ceil(T/8) and
+// T >= n - 3X (m >= 4) or n - 2(X + M) (m = 3), so S >= n whenever
+// 11 * #{positions whose key hash was seen before} <= n.
+__device__ __forceinline__ bool build_index(const Smem& S, uint32_t n, uint32_t P, const EncArgs& a,
+                                            uint32_t lane, uint32_t& nruns) {
+  const uint8_t* data = S.data;
   const uint32_t hb = a.L.hbits;
   const uint32_t B = 1u << hb;
-  uint32_t* hist = reinterpret_cast<uint32_t*>(slot);  // B u16 counters, two per word
+  const uint32_t nw = a.L.bm_words;
+  const uint32_t fb = a.L.fbits;
+  uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);  // B u16 counters, two per word
+  uint32_t* seen = reinterpret_cast<uint32_t*>(S.sorted);  // 2^fb-bit filter (index unused yet)
   for (uint32_t i = lane; i < B / 2; i += 32) hist[i] = 0;
+  for (uint32_t i = lane; i < (1u << (fb - 5)); i += 32) seen[i] = 0;
   __syncwarp();
-  // histogram of bucket sizes
-  for (uint32_t p = lane; p < P; p += 32) {
-    const uint32_t h = khash(ld32u(data, p) & a.kmask, hb);
-    atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
+  // histogram of bucket sizes + "key hash seen before" count + run starts
+  uint32_t U = 0, nr = 0;
+  const uint32_t lt = lanemask_lt();
+  for (uint32_t p0 = 0; p0 < P; p0 += 32) {
+    const uint32_t p = p0 + lane;
+    bool dup = false, rs = false;
+    if (p < P) {
+      const uint32_t key = ld32u(data, p) & a.kmask;
+      const uint32_t h = khash(key, hb);
+      atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
+      const uint32_t g = (key * 0x85EBCA6Bu) >> (32 - fb);
+      dup = atomicOr(&seen[g >> 5], 1u << (g & 31u)) & (1u << (g & 31u));
+      rs = ((key ^ (key >> 8)) & (a.kmask >> 8)) == 0 && (p == 0 || data[p - 1] != data[p]);
+    }
+    U += __popc(__ballot_sync(kFull, dup));
+    const uint32_t rb = __ballot_sync(kFull, rs);
+    const uint32_t idx = nr + __popc(rb & lt);
+    if (rs && idx < kMaxRuns) S.runs[idx] = p;
+    nr += __popc(rb);
+  }
+  nruns = nr;
+  if (11u * U <= n) return true;
+  for (uint32_t i = lane; i < nw; i += 32) {
+    S.tb[i] = 0;
+    S.mb[i] = 0;
+  }
+  for (uint32_t i = lane; i < a.C / 8; i += 32) S.flags[i] = 0;
+  for (uint32_t w = 0; w < nw; ++w) {  // change bitmap
+    const uint32_t i = (w << 5) + lane;
+    const bool ch = (i == 0) || (i >= n) || (data[i] != data[i - 1]);
+    const uint32_t b = __ballot_sync(kFull, ch);
+    if (lane == 0) S.cb[w] = b;
   }
   __syncwarp();
+  for (uint32_t j = lane; j < min(nruns, kMaxRuns); j += 32) {  // run ends
+    const uint32_t st = S.runs[j];
+    S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
+  }
   // exclusive scan of the B u16 counters, 64 per round
   uint32_t carry = 0;
   for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
@@ -177,45 +184,180 @@ __device__ __forceinline__ void build_index(const uint8_t* data, uint16_t* sorte
     carry += __shfl_sync(kFull, incl, 31);
   }
   __syncwarp();
-  // stable scatter: positions in ascending order within each bucket
-  uint16_t* cur = slot;
-  const uint32_t lt = lanemask_lt();
-  for (uint32_t p0 = 0; p0 < P; p0 += 32) {
-    const uint32_t p = p0 + lane;
-    const bool act = p < P;
-    const uint32_t h = act ? khash(ld32u(data, p) & a.kmask, hb) : 0xFFFFFFFFu;
-    const uint32_t peers = __match_any_sync(kFull, h);
-    const uint32_t rank = __popc(peers & lt);
-    const uint32_t basev = act ? cur[h] : 0;
-    if (act) sorted[basev + rank] = (uint16_t)p;
-    __syncwarp();
-    if (act && lane == 31u - __clz(peers)) cur[h] = (uint16_t)(basev + __popc(peers));
-    __syncwarp();
+  // stable scatter, 4 blocks of 32 positions per round so that the MATCH.ANY
+  // latencies overlap; cursor updates stay in position order
+  uint16_t* cur = S.slot;
+  
+  for (uint32_t p0 = 0; p0 < P; p0 += 128) {
+    uint32_t h[4], peers[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t p = p0 + 32 * u + lane;
+      h[u] = p < P ? khash(ld32u(data, p) & a.kmask, hb) : 0xFFFFFFFFu;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t p = p0 + 32 * u + lane;
+      const bool act = p < P;
+      const uint32_t basev = act ? cur[h[u]] : 0;
+      if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)p;
+      __syncwarp();
+      if (act && lane == 31u - __clz(peers[u])) cur[h[u]] = (uint16_t)(basev + __popc(peers[u]));
+      __syncwarp();
+    }
   }
-  // slot of each position (the bucket cursors are dead now)
-  for (uint32_t s = lane; s < P; s += 32) slot[sorted[s]] = (uint16_t)s;
+  // mark the first entry of every non-empty bucket (cur[h] = end of bucket h now)
+  for (uint32_t hh = lane; hh < B; hh += 32) {
+    const uint32_t st = hh ? cur[hh - 1] : 0u;
+    if (cur[hh] > st) S.sorted[st] |= kFirst;
+  }
   __syncwarp();
-  // bitmap: p has a same-key earlier position inside the window
-  for (uint32_t w = 0; w < a.L.bm_words; ++w) {
-    const uint32_t p = w * 32 + lane;
+  // slot of each position (cursors are dead now)
+  for (uint32_t s = lane; s < P; s += 32) S.slot[S.sorted[s] & kPos] = (uint16_t)s;
+  __syncwarp();
+  // candidate bitmap: nearest same-key earlier position inside the window
+  for (uint32_t w = 0; w < nw; ++w) {
+    const uint32_t p = (w << 5) + lane;
     bool has = false;
     if (p < P) {
       const uint32_t kp = ld32u(data, p) & a.kmask;
-      const uint32_t hp = khash(kp, hb);
-      for (int s = (int)slot[p] - 1; s >= 0; --s) {
-        const uint32_t q = sorted[s];
-        const uint32_t kq = ld32u(data, q) & a.kmask;
-        if (kq == kp) {
-          has = p - q <= a.W;  // nearest same-key position decides
-          break;
+      int s = S.slot[p];
+      if (!(S.sorted[s] & kFirst)) {
+        for (--s;; --s) {
+          const uint32_t e = S.sorted[s];
+          const uint32_t q = e & kPos;
+          if ((ld32u(data, q) & a.kmask) == kp) {
+            has = p - q <= a.W;
+            break;
+          }
+          if (e & kFirst) break;
         }
-        if (khash(kq, hb) != hp) break;
       }
     }
     const uint32_t b = __ballot_sync(kFull, has);
-    if (lane == 0) bm[w] = b;
+    if (lane == 0) S.cand[w] = b;
   }
   __syncwarp();
+  return false;
+}
+
+// ---- a3: longest, then nearest, capped match at p ------------------------------
+// Run-aware exact search for a position p whose key is one repeated byte b and
+// whose whole prefix lies in the window.  Every same-key candidate lies in a run
+// of b; with r = min(run length at p, cap), a candidate q with run length
+// RL(q) != r matches min(r, RL(q)) bytes and one with RL(q) == r matches
+// r + (common prefix after both runs).  So in an earlier run [s, e) of b the
+// best candidate, and the nearest among equals, is q = e - r when e - s >= r,
+// else q = s with length e - s; inside p's own run it is d = 1 with length r.
+// One lane per earlier run therefore decides the whole chunk history.
+__device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, uint32_t n,
+                                                    uint32_t cap, uint32_t kp, uint32_t nruns,
+                                                    const EncArgs& a, uint32_t lane) {
+  const uint8_t* data = S.data;
+  const uint32_t b = kp & 0xFFu;
+  const uint32_t r = run_len(S.cb, p, cap);  // >= k
+  uint32_t best = 0;
+  if (p >= 1 && data[p - 1] == b && r >= a.m) best = (r << 16) | 0xFFFFu;  // d = 1
+  for (uint32_t j0 = 0; j0 < nruns; j0 += 32) {
+    const uint32_t j = j0 + lane;
+    uint32_t pk = 0;
+    if (j < nruns) {
+      const uint32_t rr = S.runs[j];
+      const uint32_t st = rr & 0xFFFFu, e = rr >> 16;
+      if (data[st] == b) {
+        const bool reach = e - st >= r;
+        const uint32_t q = reach ? e - r : st;
+        if (q < p) {
+          const uint32_t l = !reach ? e - st : (r < cap ? r + lcp16(data, p + r, e, cap - r) : cap);
+          if (l >= a.m) pk = (l << 16) | (0xFFFFu - (p - q - 1));
+        }
+      }
+    }
+    best = max(best, __reduce_max_sync(kFull, pk));
+  }
+  return best;
+}
+
+// Returns (len << 16) | (0xFFFF - (d-1)), or 0 when no candidate reaches m.
+__device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32_t n,
+                                               uint32_t nruns, const EncArgs& a, uint32_t lane) {
+  const uint8_t* data = S.data;
+  const uint32_t cap = min(a.M, n - p);  // p < n - m + 1  =>  cap >= m >= k
+  const uint32_t kp = ld32u(data, p) & a.kmask;
+  const bool prun = ((kp ^ (kp >> 8)) & (a.kmask >> 8)) == 0;  // key = one repeated byte
+  const bool all_in_window = p <= a.W;
+  if (prun && all_in_window && nruns <= kMaxRuns)
+    return best_match_runs(S, p, n, cap, kp, nruns, a, lane);
+  // run shortcut for the generic path (window smaller than the prefix / many runs)
+  const uint32_t rp = prun ? run_len(S.cb, p, cap) : 0u;
+  uint32_t best = 0, blen = 0;
+  int sb = (int)S.slot[p] - 1;  // the walk only asks at positions with a candidate
+  for (;; sb -= 32) {
+    const int s = sb - (int)lane;
+    uint32_t e = kFirst, q = 0;
+    bool ok = s >= 0;
+    if (ok) {
+      e = S.sorted[s];
+      q = e & kPos;
+      ok = all_in_window || p - q <= a.W;
+    }
+    // lanes up to and including the bucket's first entry, and inside the window
+    const uint32_t m_first = __ballot_sync(kFull, ok && (e & kFirst));
+    const uint32_t m_stop = __ballot_sync(kFull, !ok);
+    uint32_t lim = 32;
+    if (m_first) lim = (uint32_t)__ffs(m_first);
+    if (m_stop) lim = min(lim, (uint32_t)(__ffs(m_stop) - 1));
+    uint32_t pk = 0;
+    if (lane < lim && (blen == 0 || data[q + blen] == data[p + blen])) {
+      uint32_t l;
+      if (rp) {
+        if ((ld32u(data, q) & a.kmask) != kp) {
+          l = 0;  // hash collision
+        } else {
+          const uint32_t rq = run_len(S.cb, q, cap);
+          l = rq != rp ? min(rp, rq) : (rp < cap ? rp + lcp16(data, p + rp, q + rp, cap - rp) : cap);
+        }
+      } else {
+        l = lcp16(data, p, q, cap);
+      }
+      if (l >= a.m) pk = (l << 16) | (0xFFFFu - (p - q - 1));
+    }
+    best = max(best, __reduce_max_sync(kFull, pk));
+    blen = best >> 16;
+    if (blen >= cap || lim < 32) break;
+  }
+  return best;
+}
+
+// ---- a5: parallel encode of the recorded parse into the staging buffer --------
+__device__ __forceinline__ void encode_tokens(const Smem& S, uint32_t n, uint32_t m, uint8_t* ob,
+                                              uint32_t lane) {
+  const uint32_t lt = lanemask_lt();
+  uint32_t carryT = 0, carryM = 0;
+  const uint32_t nwords = (n + 31) >> 5;
+  for (uint32_t w = 0; w < nwords; ++w) {
+    const uint32_t tw = S.tb[w], mw = S.mb[w];
+    const uint32_t p = (w << 5) + lane;
+    if ((tw >> lane) & 1u) {
+      const uint32_t j = carryT + __popc(tw & lt);
+      const uint32_t mbef = carryM + __popc(mw & lt);
+      const uint32_t pos = j + 2 * mbef + (j >> 3) + 1;
+      if ((j & 7u) == 0) ob[pos - 1] = S.flags[j >> 3];
+      if ((mw >> lane) & 1u) {
+        const uint32_t dm1 = S.slot[p], lm = S.slot[p + 1];
+        ob[pos] = (uint8_t)(dm1 & 0xFF);
+        ob[pos + 1] = (uint8_t)(dm1 >> 8);
+        ob[pos + 2] = (uint8_t)lm;
+      } else {
+        ob[pos] = S.data[p];
+      }
+    }
+    carryT += __popc(tw);
+    carryM += __popc(mw);
+  }
+  (void)m;
 }
 
 __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const EncArgs a) {
@@ -223,10 +365,18 @@ __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const Enc
   const uint32_t lane = threadIdx.x & 31u;
   const uint32_t warp = threadIdx.x >> 5;
   uint8_t* base = smem + (size_t)warp * a.L.per_warp;
-  uint8_t* data = base;
-  uint16_t* sorted = reinterpret_cast<uint16_t*>(base + a.L.off_sorted);
-  uint16_t* slot = reinterpret_cast<uint16_t*>(base + a.L.off_slot);
-  uint32_t* bm = reinterpret_cast<uint32_t*>(base + a.L.off_bm);
+  Smem S;
+  S.data = base;
+  S.sorted = reinterpret_cast<uint16_t*>(base + a.L.off_sorted);
+  S.slot = reinterpret_cast<uint16_t*>(base + a.L.off_slot);
+  uint32_t* bms = reinterpret_cast<uint32_t*>(base + a.L.off_bm);
+  const uint32_t nw = a.L.bm_words;
+  S.cand = bms;
+  S.cb = bms + nw;
+  S.tb = bms + 2 * nw;
+  S.mb = bms + 3 * nw;
+  S.flags = reinterpret_cast<uint8_t*>(bms + 4 * nw);
+  S.runs = reinterpret_cast<uint32_t*>(S.flags + align_up(a.C / 8, 4));
   uint64_t* bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
 
   if (lane == 0) {
@@ -251,56 +401,95 @@ __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const Enc
     const uint32_t n16 = n & ~15u;
     if (lane == 0 && n16) {
       mbar_arrive_expect_tx(bar, n16);
-      tma_bulk_g2s(data, src, n16, bar);
+      tma_bulk_g2s(S.data, src, n16, bar);
     }
-    for (uint32_t i = n16 + lane; i < n; i += 32) data[i] = src[i];
-    for (uint32_t i = n + lane; i < align_up(n, 16) + 16; i += 32) data[i] = 0;
+    for (uint32_t i = n16 + lane; i < n; i += 32) S.data[i] = src[i];
+    for (uint32_t i = n + lane; i < align_up(n, 16) + 32; i += 32) S.data[i] = 0;
     if (n16) {
       mbar_wait_parity(bar, phase);
       phase ^= 1u;
     }
     __syncwarp();
 
-    // ---- a3 index
     const uint32_t P = n >= a.m ? n - a.m + 1 : 0;  // positions that can start a match
-    build_index(data, sorted, slot, bm, n, P, a, lane);
+    uint32_t nruns = 0;
+    bool raw = build_index(S, n, P, a, lane, nruns);
 
-    // ---- a3/a4/a5: greedy walk + encode
-    uint8_t* out = a.slots + lo;
-    EncState e{0, 0, 0, 0};
-    bool raw = false;
+    // ---- a3/a4: greedy walk, recording the parse (bitmap words and the flag
+    // byte of the current group accumulate in registers; lane 0 stores them)
+    uint32_t T = 0, Mt = 0;
     uint32_t p = 0;
-    while (p < n) {
+    uint32_t cw = 0, acc_t = 0, acc_m = 0, gcur = 0, acc_f = 0;
+    while (!raw && p < n) {
       uint32_t bits = 0;
-      if (p < P) bits = __funnelshift_r(bm[p >> 5], bm[(p >> 5) + 1], p & 31u);
-      if (bits == 0) {
-        const uint32_t L = min(32u, n - p);
-        emit_literals(out, data, p, L, n, e, lane);
+      if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
+      const uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
+      const uint32_t w = p >> 5, sh = p & 31u;
+      if (w != cw) {
+        if (lane == 0) {
+          S.tb[cw] = acc_t;
+          S.mb[cw] = acc_m;
+        }
+        cw = w;
+        acc_t = acc_m = 0;
+      }
+      if (L) {  // run of literals
+        const uint32_t mask = L >= 32 ? 0xFFFFFFFFu : ((1u << L) - 1u);
+        acc_t |= mask << sh;
+        if (sh + L > 32) {
+          if (lane == 0) {
+            S.tb[cw] = acc_t;
+            S.mb[cw] = acc_m;
+          }
+          cw = w + 1;
+          acc_t = mask >> (32 - sh);
+          acc_m = 0;
+        }
+        T += L;
         p += L;
       } else {
-        const uint32_t f = (uint32_t)(__ffs(bits) - 1);
-        if (f) {
-          emit_literals(out, data, p, f, n, e, lane);
-          p += f;
-        } else {
-          const uint32_t r = best_match(data, sorted, slot, p, n, a, lane);
-          const uint32_t l = r >> 16;
-          if (l >= a.m) {
-            emit_match(out, 0xFFFFu - (r & 0xFFFFu) + 1, l, a.m, n, e, lane);
-            p += l;
-          } else {
-            emit_literals(out, data, p, 1, n, e, lane);
-            p += 1;
+        const uint32_t r = best_match(S, p, n, nruns, a, lane);
+        const uint32_t l = r >> 16;
+        acc_t |= 1u << sh;
+        if (l >= a.m) {
+          acc_m |= 1u << sh;
+          if (lane == 0) {
+            S.slot[p] = (uint16_t)(0xFFFFu - (r & 0xFFFFu));  // d - 1
+            S.slot[p + 1] = (uint16_t)(l - a.m);
           }
+          if ((T >> 3) != gcur) {
+            if (lane == 0 && acc_f) S.flags[gcur] = (uint8_t)acc_f;
+            gcur = T >> 3;
+            acc_f = 0;
+          }
+          acc_f |= 1u << (T & 7u);
+          Mt += 1;
+          p += l;
+        } else {
+          p += 1;
         }
+        T += 1;
       }
-      if (e.opos >= n) {
-        raw = true;  // stream not shorter than the chunk: stored raw (R9)
-        break;
-      }
+      if (T + 2 * Mt + ((T + 7) >> 3) >= n) raw = true;  // not shorter than the chunk (R9)
     }
-    if (!raw && e.cnt != 0 && lane == 0) out[e.fpos] = (uint8_t)e.fbits;
-    if (lane == 0) a.sizes[c] = raw ? n : e.opos;
+    if (!raw && lane == 0) {
+      S.tb[cw] = acc_t;
+      S.mb[cw] = acc_m;
+      if (acc_f) S.flags[gcur] = (uint8_t)acc_f;
+    }
+    __syncwarp();
+    uint32_t Sz = n;
+    if (!raw) {
+      Sz = T + 2 * Mt + ((T + 7) >> 3);
+      uint8_t* ob = reinterpret_cast<uint8_t*>(S.sorted);  // the index is dead now
+      encode_tokens(S, n, a.m, ob, lane);
+      __syncwarp();
+      uint8_t* out = a.slots + lo;
+      const uint32_t n16o = align_up(Sz, 16);
+      for (uint32_t i = lane * 16; i < n16o; i += 32 * 16)
+        *reinterpret_cast<uint4*>(out + i) = *reinterpret_cast<const uint4*>(ob + i);
+    }
+    if (lane == 0) a.sizes[c] = Sz;
     __syncwarp();
   }
 }

@@ -71,7 +71,7 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
 
 // ---- encode kernel shared-memory layout (one region per warp = per chunk) ---
 struct EncLayout {
-  uint32_t off_sorted, off_slot, off_bm, off_mbar, per_warp, hbits, bm_words;
+  uint32_t off_sorted, off_slot, off_bm, off_mbar, per_warp, hbits, bm_words, fbits;
 };
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
@@ -83,18 +83,23 @@ __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
 __host__ __device__ inline EncLayout enc_layout(uint32_t C) {
   EncLayout L;
   L.hbits = enc_hash_bits(C);
+  L.fbits = 5;  // raw pre-filter: 2^fbits bits inside the 2C-byte index region, <= 2^15
+  while ((2u << L.fbits) <= 16 * C && L.fbits < 15) ++L.fbits;
   uint32_t B = 1u << L.hbits;
-  uint32_t o = align_up(C + 16, 16);  // chunk bytes + zero pad for unaligned word loads
+  uint32_t o = align_up(C, 16) + 32;  // chunk bytes + zero pad for 16-byte compares
   L.off_sorted = o;
   o = align_up(o + 2 * C, 16);  // u16 positions grouped by hash bucket, ascending
   L.off_slot = o;
   o = align_up(o + 2 * (C > B ? C : B), 16);  // u16 slot of each position (histogram before)
   L.off_bm = o;
-  L.bm_words = C / 32 + 2;
-  o = align_up(o + 4 * L.bm_words, 16);  // candidate bitmap (1 bit per position)
+  L.bm_words = (C + 31) / 32 + 1;  // +1: two-word funnel reads at the last position
+  // four bitmaps (candidate, byte-change, token start, match), group flag bytes
+  // (C/8) and the run list (32 entries); sized so that 10 warps (chunks) fit one
+  // SM at C = 4096
+  o = align_up(o + 4 * 4 * L.bm_words + align_up(C / 8, 4) + 4 * 32, 16);
   L.off_mbar = o;
   o += 16;
-  L.per_warp = align_up(o, 128);
+  L.per_warp = align_up(o, 16);
   return L;
 }
 

@@ -82,6 +82,21 @@ def _adversarial():
     yield "binary", rng.integers(0, 2, 4096 * 6, dtype=np.uint8)
     yield "quaternary", rng.integers(0, 4, 4096 * 6, dtype=np.uint8) + 0x61
     yield "runs", np.repeat(rng.integers(0, 3, 4000, dtype=np.uint8), rng.integers(1, 40, 4000))[: 4096 * 8]
+    # run structure (exercises the run-aware search and its >64-runs fallback)
+    vals = rng.integers(0, 3, 3000, dtype=np.uint8)
+    lens = rng.integers(1, 300, 3000)
+    yield "runs_long_3vals", np.repeat(vals, lens)[: 4096 * 8 + 100]
+    yield "runs_short_many", np.repeat(rng.integers(0, 2, 6000, dtype=np.uint8), rng.integers(3, 9, 6000))[: 4096 * 6]
+    zr = []
+    for k in range(400):
+        zr.append(np.zeros(int(rng.integers(4, 600)), np.uint8))
+        zr.append(rng.integers(0, 256, int(rng.integers(1, 20)), dtype=np.uint8))
+    yield "zero_runs_mixed_tails", np.concatenate(zr)[: 4096 * 10 + 7]
+    pat = []
+    for k in range(600):  # runs followed by repeated tails: exact-RL candidates with continuations
+        pat.append(np.full(int(rng.integers(4, 40)), int(rng.integers(0, 2)), np.uint8))
+        pat.append(np.frombuffer(b"xyz" if k % 3 else b"xyw", np.uint8))
+    yield "runs_with_shared_tails", np.concatenate(pat)[: 4096 * 6]
     yield "tiny1", np.array([7], np.uint8)
     yield "tiny5", np.frombuffer(b"aaaaa", np.uint8).copy()
 
@@ -92,7 +107,7 @@ def test_adversarial_bitexact(lzr, ref, name, x):
 
 
 @pytest.mark.parametrize("C,W,m,M", [
-    (4096, 4096, 3, 258), (4096, 4096, 5, 40), (4096, 4096, 4, 4), (4096, 4096, 4, 5),
+    (4096, 4096, 3, 258), (4096, 4096, 5, 40), (4096, 4096, 3, 3), (4096, 4096, 9, 12), (4096, 4096, 4, 4), (4096, 4096, 4, 5),
     (4096, 1000, 4, 259), (4096, 1, 4, 259), (4096, 2, 3, 100), (4096, 33, 6, 261),
     (16, 16, 3, 258), (16, 5, 4, 259), (48, 48, 4, 259), (528, 300, 4, 20),
     (8192, 8192, 4, 259), (16384, 16384, 4, 259), (32768, 32768, 4, 259),
