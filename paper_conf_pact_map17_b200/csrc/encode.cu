@@ -80,6 +80,25 @@ __device__ __forceinline__ uint32_t lcp16(const uint8_t* d, uint32_t a, uint32_t
   return maxlen;
 }
 
+// lcp16 for the common call (p-side start fixed for all lanes): the first 16
+// p-side bytes are preloaded once per search (pw).
+__device__ __forceinline__ uint32_t lcp16_pre(const uint8_t* d, const uint32_t (&pw)[4], uint32_t p,
+                                              uint32_t q, uint32_t maxlen) {
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(d);
+  const uint32_t sb = (q & 3u) << 3, ib = q >> 2;
+  const uint32_t b0 = w[ib], b1 = w[ib + 1], b2 = w[ib + 2], b3 = w[ib + 3], b4 = w[ib + 4];
+  const uint32_t x0 = pw[0] ^ __funnelshift_r(b0, b1, sb);
+  const uint32_t x1 = pw[1] ^ __funnelshift_r(b1, b2, sb);
+  const uint32_t x2 = pw[2] ^ __funnelshift_r(b2, b3, sb);
+  const uint32_t x3 = pw[3] ^ __funnelshift_r(b3, b4, sb);
+  const uint64_t lo = ((uint64_t)x1 << 32) | x0, hi = ((uint64_t)x3 << 32) | x2;
+  uint32_t l;
+  if (lo) l = (uint32_t)(__ffsll((long long)lo) - 1) >> 3;
+  else if (hi) l = 8 + ((uint32_t)(__ffsll((long long)hi) - 1) >> 3);
+  else l = maxlen > 16 ? 16 + lcp16(d, p + 16, q + 16, maxlen - 16) : 16;
+  return l < maxlen ? l : maxlen;
+}
+
 // min(run length of the byte at p, lim): distance to the next set bit of the
 // change bitmap cb (bit i = x[i] != x[i-1]; set for i >= n).
 __device__ __forceinline__ uint32_t run_len(const uint32_t* cb, uint32_t p, uint32_t lim) {
@@ -104,8 +123,9 @@ struct Smem {
                      // after the walk: (d-1) at a match start, (l-m) right after it
   uint32_t* cand;    // 1: a same-key position exists inside the window
   uint32_t* cb;      // 1: byte differs from the previous one (run boundaries)
-  uint32_t* tb;      // 1: token starts here
-  uint32_t* mb;      // 1: the token here is a match
+  uint32_t* tg;      // match toggles: bit s+1 and bit s+l for a match (s, l);
+                     // prefix parity = "inside a match", so token starts and
+                     // match starts follow without recording literals
   uint8_t* flags;    // flag byte of each group of 8 tokens
   uint32_t* runs;    // (end << 16) | start of every run of >= k equal bytes (first kMaxRuns)
 };
@@ -152,8 +172,8 @@ __device__ __forceinline__ bool build_index(const Smem& S, uint32_t n, uint32_t 
   nruns = nr;
   if (11u * U <= n) return true;
   for (uint32_t i = lane; i < nw; i += 32) {
-    S.tb[i] = 0;
-    S.mb[i] = 0;
+    S.tg[i] = 0;
+    S.cand[i] = 0;
   }
   for (uint32_t i = lane; i < a.C / 8; i += 32) S.flags[i] = 0;
   for (uint32_t w = 0; w < nw; ++w) {  // change bitmap
@@ -214,30 +234,27 @@ __device__ __forceinline__ bool build_index(const Smem& S, uint32_t n, uint32_t 
     if (cur[hh] > st) S.sorted[st] |= kFirst;
   }
   __syncwarp();
-  // slot of each position (cursors are dead now)
-  for (uint32_t s = lane; s < P; s += 32) S.slot[S.sorted[s] & kPos] = (uint16_t)s;
-  __syncwarp();
-  // candidate bitmap: nearest same-key earlier position inside the window
-  for (uint32_t w = 0; w < nw; ++w) {
-    const uint32_t p = (w << 5) + lane;
-    bool has = false;
-    if (p < P) {
-      const uint32_t kp = ld32u(data, p) & a.kmask;
-      int s = S.slot[p];
-      if (!(S.sorted[s] & kFirst)) {
-        for (--s;; --s) {
-          const uint32_t e = S.sorted[s];
-          const uint32_t q = e & kPos;
-          if ((ld32u(data, q) & a.kmask) == kp) {
-            has = p - q <= a.W;
-            break;
-          }
-          if (e & kFirst) break;
+  // slot of each position (cursors are dead now) and the candidate bitmap: the
+  // nearest same-key earlier position is the nearest same-key entry below in
+  // the bucket; it decides whether a candidate lies inside the window
+  for (uint32_t sl = lane; sl < P; sl += 32) {
+    const uint32_t e = S.sorted[sl];
+    const uint32_t q = e & kPos;
+    S.slot[q] = (uint16_t)sl;
+    if (!(e & kFirst)) {
+      const uint32_t kq = ld32u(data, q) & a.kmask;
+      bool has = false;
+      for (uint32_t s2 = sl - 1;; --s2) {
+        const uint32_t e2 = S.sorted[s2];
+        const uint32_t q2 = e2 & kPos;
+        if ((ld32u(data, q2) & a.kmask) == kq) {
+          has = q - q2 <= a.W;
+          break;
         }
+        if (e2 & kFirst) break;
       }
+      if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
     }
-    const uint32_t b = __ballot_sync(kFull, has);
-    if (lane == 0) S.cand[w] = b;
   }
   __syncwarp();
   return false;
@@ -292,6 +309,16 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
     return best_match_runs(S, p, n, cap, kp, nruns, a, lane);
   // run shortcut for the generic path (window smaller than the prefix / many runs)
   const uint32_t rp = prun ? run_len(S.cb, p, cap) : 0u;
+  uint32_t pw[4];
+  {
+    const uint32_t* w = reinterpret_cast<const uint32_t*>(data);
+    const uint32_t sa = (p & 3u) << 3, ia = p >> 2;
+    const uint32_t a0 = w[ia], a1 = w[ia + 1], a2 = w[ia + 2], a3 = w[ia + 3], a4 = w[ia + 4];
+    pw[0] = __funnelshift_r(a0, a1, sa);
+    pw[1] = __funnelshift_r(a1, a2, sa);
+    pw[2] = __funnelshift_r(a2, a3, sa);
+    pw[3] = __funnelshift_r(a3, a4, sa);
+  }
   uint32_t best = 0, blen = 0;
   int sb = (int)S.slot[p] - 1;  // the walk only asks at positions with a candidate
   for (;; sb -= 32) {
@@ -320,7 +347,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
           l = rq != rp ? min(rp, rq) : (rp < cap ? rp + lcp16(data, p + rp, q + rp, cap - rp) : cap);
         }
       } else {
-        l = lcp16(data, p, q, cap);
+        l = lcp16_pre(data, pw, p, q, cap);
       }
       if (l >= a.m) pk = (l << 16) | (0xFFFFu - (p - q - 1));
     }
@@ -332,13 +359,31 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 }
 
 // ---- a5: parallel encode of the recorded parse into the staging buffer --------
-__device__ __forceinline__ void encode_tokens(const Smem& S, uint32_t n, uint32_t m, uint8_t* ob,
-                                              uint32_t lane) {
+// inside(t) = parity of match toggles at positions <= t; token starts are the
+// positions not inside a match, match starts s have inside(s) = 0, inside(s+1) = 1.
+__device__ __forceinline__ uint32_t prefix_parity(uint32_t x) {
+  x ^= x << 1;
+  x ^= x << 2;
+  x ^= x << 4;
+  x ^= x << 8;
+  x ^= x << 16;
+  return x;
+}
+
+__device__ __forceinline__ void encode_tokens(const Smem& S, uint32_t n, uint8_t* ob, uint32_t lane) {
   const uint32_t lt = lanemask_lt();
-  uint32_t carryT = 0, carryM = 0;
+  uint32_t carryT = 0, carryM = 0, par = 0;
   const uint32_t nwords = (n + 31) >> 5;
+  uint32_t tg_next = S.tg[0];
   for (uint32_t w = 0; w < nwords; ++w) {
-    const uint32_t tw = S.tb[w], mw = S.mb[w];
+    const uint32_t tgw = tg_next;
+    tg_next = S.tg[w + 1];
+    const uint32_t inside = prefix_parity(tgw) ^ (0u - par);
+    par = inside >> 31;
+    const uint32_t next0 = par ^ (tg_next & 1u);
+    const uint32_t valid = (n - (w << 5)) >= 32 ? 0xFFFFFFFFu : ((1u << (n - (w << 5))) - 1u);
+    const uint32_t tw = ~inside & valid;
+    const uint32_t mw = ~inside & ((inside >> 1) | (next0 << 31)) & valid;
     const uint32_t p = (w << 5) + lane;
     if ((tw >> lane) & 1u) {
       const uint32_t j = carryT + __popc(tw & lt);
@@ -357,7 +402,6 @@ __device__ __forceinline__ void encode_tokens(const Smem& S, uint32_t n, uint32_
     carryT += __popc(tw);
     carryM += __popc(mw);
   }
-  (void)m;
 }
 
 __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const EncArgs a) {
@@ -373,8 +417,7 @@ __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const Enc
   const uint32_t nw = a.L.bm_words;
   S.cand = bms;
   S.cb = bms + nw;
-  S.tb = bms + 2 * nw;
-  S.mb = bms + 3 * nw;
+  S.tg = bms + 2 * nw;
   S.flags = reinterpret_cast<uint8_t*>(bms + 4 * nw);
   S.runs = reinterpret_cast<uint32_t*>(S.flags + align_up(a.C / 8, 4));
   uint64_t* bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
@@ -415,45 +458,29 @@ __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const Enc
     uint32_t nruns = 0;
     bool raw = build_index(S, n, P, a, lane, nruns);
 
-    // ---- a3/a4: greedy walk, recording the parse (bitmap words and the flag
-    // byte of the current group accumulate in registers; lane 0 stores them)
+    // ---- a3/a4: greedy walk.  Only matches are recorded (toggles, (d-1), (l-m));
+    // literal runs just advance p and the token count T; the flag byte of the
+    // current group of 8 tokens accumulates in a register.
     uint32_t T = 0, Mt = 0;
     uint32_t p = 0;
-    uint32_t cw = 0, acc_t = 0, acc_m = 0, gcur = 0, acc_f = 0;
+    uint32_t gcur = 0, acc_f = 0;
     while (!raw && p < n) {
       uint32_t bits = 0;
       if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
-      const uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
-      const uint32_t w = p >> 5, sh = p & 31u;
-      if (w != cw) {
-        if (lane == 0) {
-          S.tb[cw] = acc_t;
-          S.mb[cw] = acc_m;
-        }
-        cw = w;
-        acc_t = acc_m = 0;
-      }
-      if (L) {  // run of literals
-        const uint32_t mask = L >= 32 ? 0xFFFFFFFFu : ((1u << L) - 1u);
-        acc_t |= mask << sh;
-        if (sh + L > 32) {
-          if (lane == 0) {
-            S.tb[cw] = acc_t;
-            S.mb[cw] = acc_m;
-          }
-          cw = w + 1;
-          acc_t = mask >> (32 - sh);
-          acc_m = 0;
-        }
+      if (bits == 0) {  // 32 (or the rest) literals
+        const uint32_t L = min(32u, n - p);
         T += L;
         p += L;
       } else {
+        const uint32_t f = (uint32_t)(__ffs(bits) - 1);  // literals before the candidate
+        T += f;
+        p += f;
         const uint32_t r = best_match(S, p, n, nruns, a, lane);
         const uint32_t l = r >> 16;
-        acc_t |= 1u << sh;
         if (l >= a.m) {
-          acc_m |= 1u << sh;
           if (lane == 0) {
+            atomicOr(&S.tg[(p + 1) >> 5], 1u << ((p + 1) & 31u));
+            atomicOr(&S.tg[(p + l) >> 5], 1u << ((p + l) & 31u));
             S.slot[p] = (uint16_t)(0xFFFFu - (r & 0xFFFFu));  // d - 1
             S.slot[p + 1] = (uint16_t)(l - a.m);
           }
@@ -472,17 +499,13 @@ __global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const Enc
       }
       if (T + 2 * Mt + ((T + 7) >> 3) >= n) raw = true;  // not shorter than the chunk (R9)
     }
-    if (!raw && lane == 0) {
-      S.tb[cw] = acc_t;
-      S.mb[cw] = acc_m;
-      if (acc_f) S.flags[gcur] = (uint8_t)acc_f;
-    }
+    if (!raw && lane == 0 && acc_f) S.flags[gcur] = (uint8_t)acc_f;
     __syncwarp();
     uint32_t Sz = n;
     if (!raw) {
       Sz = T + 2 * Mt + ((T + 7) >> 3);
       uint8_t* ob = reinterpret_cast<uint8_t*>(S.sorted);  // the index is dead now
-      encode_tokens(S, n, a.m, ob, lane);
+      encode_tokens(S, n, ob, lane);
       __syncwarp();
       uint8_t* out = a.slots + lo;
       const uint32_t n16o = align_up(Sz, 16);
