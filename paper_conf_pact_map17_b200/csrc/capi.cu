@@ -3,6 +3,7 @@
 // the host-buffer end-to-end pipeline.  No device memory is allocated here.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <mutex>
@@ -43,6 +44,17 @@ cudaError_t dev_info(DevInfo* out) {
 
 bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
+// Warps cooperating on one chunk (K).  LZR_ENCODE_WARPS=1..4 overrides (tuning).
+uint32_t enc_warps_per_chunk(uint32_t C) {
+  static int env = -1;
+  if (env < 0) {
+    const char* e = getenv("LZR_ENCODE_WARPS");
+    env = (e && *e >= '1' && *e <= '4') ? (*e - '0') : 0;
+  }
+  if (env > 0) return (uint32_t)env;
+  return C >= 1024 ? 4u : 1u;
+}
+
 }  // namespace
 
 WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
@@ -51,7 +63,7 @@ WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
   const size_t N = (n_bytes + C - 1) / C;
   w.ctrl_off = 0;
   w.slots_off = 256;
-  w.scan_off = w.slots_off + align_up_z(N * C, 256);
+  w.scan_off = w.slots_off + align_up_z(N * 2 * C, 256);  // per chunk: (d-1) scratch, then stream
   w.total = w.scan_off + scan_ws_bytes(N);
   return w;
 }
@@ -128,10 +140,10 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.M = p->max_match;
   a.kbytes = p->min_match < 4 ? p->min_match : 4;
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
-  a.L = enc_layout(p->chunk_size);
+  a.L = enc_layout(p->chunk_size, enc_warps_per_chunk(p->chunk_size));
   // positions are 15-bit in the index (bit 15 marks bucket starts) and one
   // chunk's index must fit one CTA's shared memory
-  if (p->chunk_size > 32768 || (int)a.L.per_warp > di.smem_optin) return LZR_ERR_UNSUPPORTED;
+  if (p->chunk_size > 32768 || (int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;
   uint8_t* ws = (uint8_t*)d_workspace;
   a.slots = ws + w.slots_off;
   a.sizes = d_sizes;
@@ -167,7 +179,8 @@ int lzr_compress_compact(const void* d_in, size_t n_bytes, const lzr_params* p, 
   uint8_t* ws = (uint8_t*)d_workspace;
   if (launch_scan(d_sizes, N, 0, d_offsets, d_total, ws + w.scan_off, s, &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
-  if (launch_compact((const uint8_t*)d_in, n_bytes, p->chunk_size, ws + w.slots_off, d_sizes,
+  if (launch_compact((const uint8_t*)d_in, n_bytes, p->chunk_size, ws + w.slots_off,
+                     2 * (size_t)p->chunk_size, d_sizes,
                      d_offsets, (uint8_t*)d_out, di.sm_count, s, &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;

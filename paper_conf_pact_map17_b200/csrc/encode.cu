@@ -1,33 +1,36 @@
-// encode.cu -- the compression hot path on sm_100a: one warp per chunk.
+// encode.cu -- the compression hot path on sm_100a: K warps per chunk.
 //
 // Steps (§3.2(2) "The GPU allocates multiple
 // threads for each chunk. Each stage performs its own LZ compression algorithm
-// with its own history buffer and look-ahead buffer."):
+// with its own history buffer and look-ahead buffer. Adjacent threads inspect
+// overlapping regions by the size of the history buffer."):
 //   a2  stage the chunk (= its whole history window, R2) into shared memory with
 //       a 1-D bulk TMA copy (cp.async.bulk + mbarrier).
-//   a3  index: exact candidates of p are the earlier positions with the same
-//       first k = min(m,4) bytes (a match of length >= m >= k starts with them).
-//       The warp counting-sorts positions by a hash of that key into buckets
-//       kept in ascending position order (stable scatter, MATCH.ANY ranks); bit
-//       15 of an entry marks the first entry of its bucket.  A per-position bit
-//       says whether a same-key position exists inside the window, and a
-//       "byte changes here" bitmap gives run lengths in O(1) for the run
-//       shortcut below.
-//   a3  longest match at a token start p: the 32 lanes take the 32 nearest
-//       candidates (slots below p's own), compute the capped common-prefix
-//       length with 16-byte compares (or, when both sides start inside runs of
-//       the same byte, straight from the two run lengths), pack
-//       (len << 16 | 0xFFFF - (d-1)) and reduce with REDUX.MAX = "longest, then
-//       nearest" (R6, R7).  A farther candidate must also match the byte at the
-//       best length so far to be strictly longer, so most cost one compare.
-//       Stop at the cap (exact: nothing beats it) or when bucket/window end.
-//   a4  greedy walk (R8): literal runs advance up to 32 positions per step via
-//       the candidate bitmap; the walk only records token starts, match bits,
-//       (d-1) and (l-m) in place and keeps the running stream size, so a chunk
-//       whose stream reaches n bytes is stored raw (R9) without encoding.
-//   a5  encode (R1) in parallel over positions: token index and match count by
-//       ballot/popc prefix sums give every token's output byte position; the
-//       stream is assembled in shared memory and written with 16-byte stores.
+//   a3  index (the group's K warps share the passes): exact candidates of p are
+//       the earlier positions with the same first k = min(m,4) bytes (a match
+//       of length >= m >= k starts with them).  Positions are counting-sorted
+//       by a hash of that key into buckets kept in ascending position order
+//       (stable scatter, MATCH.ANY ranks); bit 15 of an entry marks the first
+//       entry of its bucket.  A candidate bitmap says whether a same-key
+//       position exists inside the window; a byte-change bitmap and a run list
+//       serve the run-aware search.  A sound pre-filter proves most
+//       incompressible chunks raw before any of this.
+//   a3  longest match at a token start p (one warp): the 32 lanes take the 32
+//       nearest candidates, compute capped common-prefix lengths with 16-byte
+//       compares, pack (len << 16 | 0xFFFF - (d-1)) and reduce with REDUX.MAX =
+//       "longest, then nearest" (R6, R7); positions whose key is one repeated
+//       byte use the exact run-aware search instead.
+//   a4  greedy walk (R8), split into K speculative segments: warp k parses from
+//       k*n/K.  Greedy parses are deterministic, so two parses that share one
+//       token start coincide from there on; warp k stops at the first of its
+//       token starts that warp k+1 has also recorded, and the exact serial parse
+//       is the chain warp 0 -> warp 1 -> ... through those meeting points (the
+//       paper's overlapping per-thread regions, made exact).  The parse is kept
+//       as a token-start bitmap plus (d-1) at each match start.
+//   a5  encode (R1) in parallel over positions: a token is a match iff the next
+//       token starts more than one byte later; token index and match count by
+//       popc prefix sums give every token's byte position; the stream is staged
+//       in shared memory and written with 16-byte stores; raw fallback (R9).
 // The serial result is reproduced exactly: the best match at p depends only on
 // (chunk bytes, p, W, m, M), not on the parse.
 #include "lzr_internal.cuh"
@@ -36,13 +39,26 @@ namespace lzr {
 
 namespace {
 
-constexpr int kMaxWarps = 16;
 constexpr uint16_t kFirst = 0x8000;  // first entry of its bucket
 constexpr uint16_t kPos = 0x7FFF;
 constexpr uint32_t kMaxRuns = 32;  // runs of one byte value of length >= k, per chunk
 
+// ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K], T[K], M[K]
+constexpr int kCtrlChunk = 0, kCtrlU = 1, kCtrlRuns = 2, kCtrlProg = 4;
+
 __device__ __forceinline__ uint32_t khash(uint32_t key, uint32_t hbits) {
   return (key * 0x9E3779B1u) >> (32 - hbits);
+}
+
+__device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+__device__ __forceinline__ uint32_t ld_volatile(const uint32_t* p) {
+  return *reinterpret_cast<const volatile uint32_t*>(p);
+}
+__device__ __forceinline__ void st_volatile(uint32_t* p, uint32_t v) {
+  *reinterpret_cast<volatile uint32_t*>(p) = v;
 }
 
 // Common-prefix length of data[a..] and data[b..], capped at maxlen; 16 bytes
@@ -62,13 +78,10 @@ __device__ __forceinline__ uint32_t lcp16(const uint8_t* d, uint32_t a, uint32_t
     const uint32_t x1 = __funnelshift_r(a1, a2, sa) ^ __funnelshift_r(b1, b2, sb);
     const uint32_t x2 = __funnelshift_r(a2, a3, sa) ^ __funnelshift_r(b2, b3, sb);
     const uint32_t x3 = __funnelshift_r(a3, a4, sa) ^ __funnelshift_r(b3, b4, sb);
-    if (x0 | x1 | x2 | x3) {
-      uint32_t k, x;
-      if (x0) { k = 0; x = x0; }
-      else if (x1) { k = 4; x = x1; }
-      else if (x2) { k = 8; x = x2; }
-      else { k = 12; x = x3; }
-      l += k + ((uint32_t)(__ffs(x) - 1) >> 3);
+    const uint64_t lo = ((uint64_t)x1 << 32) | x0, hi = ((uint64_t)x3 << 32) | x2;
+    if (lo | hi) {
+      l += lo ? ((uint32_t)(__ffsll((long long)lo) - 1) >> 3)
+              : 8 + ((uint32_t)(__ffsll((long long)hi) - 1) >> 3);
       return l < maxlen ? l : maxlen;
     }
     l += 16;
@@ -116,149 +129,20 @@ __device__ __forceinline__ uint32_t run_len(const uint32_t* cb, uint32_t p, uint
   return r < lim ? r : lim;
 }
 
+// Shared memory of one group (one chunk in flight).
 struct Smem {
   uint8_t* data;
-  uint16_t* sorted;  // entries: position | kFirst; later: the output stream staging
-  uint16_t* slot;    // histogram/cursors during the sort; slot of each position;
-                     // after the walk: (d-1) at a match start, (l-m) right after it
-  uint32_t* cand;    // 1: a same-key position exists inside the window
-  uint32_t* cb;      // 1: byte differs from the previous one (run boundaries)
-  uint32_t* tg;      // match toggles: bit s+1 and bit s+l for a match (s, l);
-                     // prefix parity = "inside a match", so token starts and
-                     // match starts follow without recording literals
-  uint8_t* flags;    // flag byte of each group of 8 tokens
-  uint32_t* runs;    // (end << 16) | start of every run of >= k equal bytes (first kMaxRuns)
+  uint16_t* sorted;  // entries: position | kFirst; after the walk: output staging
+  uint16_t* slot;    // histogram/cursors during the sort; slot of each position
+  uint32_t* cand;    // 1: a same-key position exists inside the window;
+                     // after the walk: the final token-start bitmap (+ bit n)
+  uint32_t* cb;      // 1: byte differs from the previous one (run boundaries);
+                     // after the walk: match bit per token index (flag bytes)
+  uint32_t* tb;      // K token-start bitmaps, one per walk segment
+  uint32_t* runs;    // (end << 16) | start of every run of >= k equal bytes
+  uint32_t* ctrl;    // chunk, U, nruns, prog[K], sync[K], T[K], M[K]
+  uint64_t* bar;
 };
-
-// ---- a3: index ----------------------------------------------------------------
-// Returns true when the chunk is certainly stored raw (R9) and the index was not
-// built.  Sound bound: a match of length l at p makes positions p..p+l-k
-// (k = key bytes) positions with a same-key earlier occurrence, disjoint across
-// matches; with X = sum(l - 3) and T tokens, S = n - X + ceil(T/8) and
-// T >= n - 3X (m >= 4) or n - 2(X + M) (m = 3), so S >= n whenever
-// 11 * #{positions whose key hash was seen before} <= n.
-__device__ __forceinline__ bool build_index(const Smem& S, uint32_t n, uint32_t P, const EncArgs& a,
-                                            uint32_t lane, uint32_t& nruns) {
-  const uint8_t* data = S.data;
-  const uint32_t hb = a.L.hbits;
-  const uint32_t B = 1u << hb;
-  const uint32_t nw = a.L.bm_words;
-  const uint32_t fb = a.L.fbits;
-  uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);  // B u16 counters, two per word
-  uint32_t* seen = reinterpret_cast<uint32_t*>(S.sorted);  // 2^fb-bit filter (index unused yet)
-  for (uint32_t i = lane; i < B / 2; i += 32) hist[i] = 0;
-  for (uint32_t i = lane; i < (1u << (fb - 5)); i += 32) seen[i] = 0;
-  __syncwarp();
-  // histogram of bucket sizes + "key hash seen before" count + run starts
-  uint32_t U = 0, nr = 0;
-  const uint32_t lt = lanemask_lt();
-  for (uint32_t p0 = 0; p0 < P; p0 += 32) {
-    const uint32_t p = p0 + lane;
-    bool dup = false, rs = false;
-    if (p < P) {
-      const uint32_t key = ld32u(data, p) & a.kmask;
-      const uint32_t h = khash(key, hb);
-      atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
-      const uint32_t g = (key * 0x85EBCA6Bu) >> (32 - fb);
-      dup = atomicOr(&seen[g >> 5], 1u << (g & 31u)) & (1u << (g & 31u));
-      rs = ((key ^ (key >> 8)) & (a.kmask >> 8)) == 0 && (p == 0 || data[p - 1] != data[p]);
-    }
-    U += __popc(__ballot_sync(kFull, dup));
-    const uint32_t rb = __ballot_sync(kFull, rs);
-    const uint32_t idx = nr + __popc(rb & lt);
-    if (rs && idx < kMaxRuns) S.runs[idx] = p;
-    nr += __popc(rb);
-  }
-  nruns = nr;
-  if (11u * U <= n) return true;
-  for (uint32_t i = lane; i < nw; i += 32) {
-    S.tg[i] = 0;
-    S.cand[i] = 0;
-  }
-  for (uint32_t i = lane; i < a.C / 8; i += 32) S.flags[i] = 0;
-  for (uint32_t w = 0; w < nw; ++w) {  // change bitmap
-    const uint32_t i = (w << 5) + lane;
-    const bool ch = (i == 0) || (i >= n) || (data[i] != data[i - 1]);
-    const uint32_t b = __ballot_sync(kFull, ch);
-    if (lane == 0) S.cb[w] = b;
-  }
-  __syncwarp();
-  for (uint32_t j = lane; j < min(nruns, kMaxRuns); j += 32) {  // run ends
-    const uint32_t st = S.runs[j];
-    S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
-  }
-  // exclusive scan of the B u16 counters, 64 per round
-  uint32_t carry = 0;
-  for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
-    const bool act = w0 + lane < B / 2;
-    const uint32_t wv = act ? hist[w0 + lane] : 0;
-    const uint32_t c0 = wv & 0xFFFFu, sum = c0 + (wv >> 16);
-    uint32_t incl = sum;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t t = __shfl_up_sync(kFull, incl, o);
-      if ((int)lane >= o) incl += t;
-    }
-    const uint32_t excl = incl - sum + carry;
-    if (act) hist[w0 + lane] = (excl & 0xFFFFu) | ((excl + c0) << 16);
-    carry += __shfl_sync(kFull, incl, 31);
-  }
-  __syncwarp();
-  // stable scatter, 4 blocks of 32 positions per round so that the MATCH.ANY
-  // latencies overlap; cursor updates stay in position order
-  uint16_t* cur = S.slot;
-  
-  for (uint32_t p0 = 0; p0 < P; p0 += 128) {
-    uint32_t h[4], peers[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const uint32_t p = p0 + 32 * u + lane;
-      h[u] = p < P ? khash(ld32u(data, p) & a.kmask, hb) : 0xFFFFFFFFu;
-    }
-#pragma unroll
-    for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const uint32_t p = p0 + 32 * u + lane;
-      const bool act = p < P;
-      const uint32_t basev = act ? cur[h[u]] : 0;
-      if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)p;
-      __syncwarp();
-      if (act && lane == 31u - __clz(peers[u])) cur[h[u]] = (uint16_t)(basev + __popc(peers[u]));
-      __syncwarp();
-    }
-  }
-  // mark the first entry of every non-empty bucket (cur[h] = end of bucket h now)
-  for (uint32_t hh = lane; hh < B; hh += 32) {
-    const uint32_t st = hh ? cur[hh - 1] : 0u;
-    if (cur[hh] > st) S.sorted[st] |= kFirst;
-  }
-  __syncwarp();
-  // slot of each position (cursors are dead now) and the candidate bitmap: the
-  // nearest same-key earlier position is the nearest same-key entry below in
-  // the bucket; it decides whether a candidate lies inside the window
-  for (uint32_t sl = lane; sl < P; sl += 32) {
-    const uint32_t e = S.sorted[sl];
-    const uint32_t q = e & kPos;
-    S.slot[q] = (uint16_t)sl;
-    if (!(e & kFirst)) {
-      const uint32_t kq = ld32u(data, q) & a.kmask;
-      bool has = false;
-      for (uint32_t s2 = sl - 1;; --s2) {
-        const uint32_t e2 = S.sorted[s2];
-        const uint32_t q2 = e2 & kPos;
-        if ((ld32u(data, q2) & a.kmask) == kq) {
-          has = q - q2 <= a.W;
-          break;
-        }
-        if (e2 & kFirst) break;
-      }
-      if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
-    }
-  }
-  __syncwarp();
-  return false;
-}
 
 // ---- a3: longest, then nearest, capped match at p ------------------------------
 // Run-aware exact search for a position p whose key is one repeated byte b and
@@ -269,9 +153,9 @@ __device__ __forceinline__ bool build_index(const Smem& S, uint32_t n, uint32_t 
 // best candidate, and the nearest among equals, is q = e - r when e - s >= r,
 // else q = s with length e - s; inside p's own run it is d = 1 with length r.
 // One lane per earlier run therefore decides the whole chunk history.
-__device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, uint32_t n,
-                                                    uint32_t cap, uint32_t kp, uint32_t nruns,
-                                                    const EncArgs& a, uint32_t lane) {
+__device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, uint32_t cap,
+                                                    uint32_t kp, uint32_t nruns, const EncArgs& a,
+                                                    uint32_t lane) {
   const uint8_t* data = S.data;
   const uint32_t b = kp & 0xFFu;
   const uint32_t r = run_len(S.cb, p, cap);  // >= k
@@ -306,7 +190,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   const bool prun = ((kp ^ (kp >> 8)) & (a.kmask >> 8)) == 0;  // key = one repeated byte
   const bool all_in_window = p <= a.W;
   if (prun && all_in_window && nruns <= kMaxRuns)
-    return best_match_runs(S, p, n, cap, kp, nruns, a, lane);
+    return best_match_runs(S, p, cap, kp, nruns, a, lane);
   // run shortcut for the generic path (window smaller than the prefix / many runs)
   const uint32_t rp = prun ? run_len(S.cb, p, cap) : 0u;
   uint32_t pw[4];
@@ -358,181 +242,483 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   return best;
 }
 
-// ---- a5: parallel encode of the recorded parse into the staging buffer --------
-// inside(t) = parity of match toggles at positions <= t; token starts are the
-// positions not inside a match, match starts s have inside(s) = 0, inside(s+1) = 1.
-__device__ __forceinline__ uint32_t prefix_parity(uint32_t x) {
-  x ^= x << 1;
-  x ^= x << 2;
-  x ^= x << 4;
-  x ^= x << 8;
-  x ^= x << 16;
-  return x;
-}
-
-__device__ __forceinline__ void encode_tokens(const Smem& S, uint32_t n, uint8_t* ob, uint32_t lane) {
-  const uint32_t lt = lanemask_lt();
-  uint32_t carryT = 0, carryM = 0, par = 0;
-  const uint32_t nwords = (n + 31) >> 5;
-  uint32_t tg_next = S.tg[0];
-  for (uint32_t w = 0; w < nwords; ++w) {
-    const uint32_t tgw = tg_next;
-    tg_next = S.tg[w + 1];
-    const uint32_t inside = prefix_parity(tgw) ^ (0u - par);
-    par = inside >> 31;
-    const uint32_t next0 = par ^ (tg_next & 1u);
-    const uint32_t valid = (n - (w << 5)) >= 32 ? 0xFFFFFFFFu : ((1u << (n - (w << 5))) - 1u);
-    const uint32_t tw = ~inside & valid;
-    const uint32_t mw = ~inside & ((inside >> 1) | (next0 << 31)) & valid;
-    const uint32_t p = (w << 5) + lane;
-    if ((tw >> lane) & 1u) {
-      const uint32_t j = carryT + __popc(tw & lt);
-      const uint32_t mbef = carryM + __popc(mw & lt);
-      const uint32_t pos = j + 2 * mbef + (j >> 3) + 1;
-      if ((j & 7u) == 0) ob[pos - 1] = S.flags[j >> 3];
-      if ((mw >> lane) & 1u) {
-        const uint32_t dm1 = S.slot[p], lm = S.slot[p + 1];
-        ob[pos] = (uint8_t)(dm1 & 0xFF);
-        ob[pos + 1] = (uint8_t)(dm1 >> 8);
-        ob[pos + 2] = (uint8_t)lm;
-      } else {
-        ob[pos] = S.data[p];
+// ---- a4: one speculative walk segment ----------------------------------------
+// Warp k parses greedily from `start`.  Token starts go into its bitmap tbk
+// (lane 0, atomics), (d-1) into d1[s] at each match start s (global scratch in
+// the chunk's workspace slot; identical from every warp that records a token
+// at s, since the best match at s does not depend on the parse).  prog[k]: every token start of warp k below prog[k] is
+// recorded.  A warp with a successor stops at the first of its token starts x
+// that the successor has recorded (x < prog[k+1]); sync[k] = x, or n if it ran
+// to the end.
+template <int K>
+__device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
+                                             uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
+                                             const EncArgs& a, uint32_t lane) {
+  const uint32_t nw = a.L.bm_words;
+  uint32_t* tbk = S.tb + k * nw;
+  const uint32_t* tbn = S.tb + (k + 1) * nw;  // successor's bitmap (k < K-1 only)
+  uint32_t* prog = S.ctrl + kCtrlProg;
+  uint32_t* sync = prog + K;
+  uint32_t p = start;
+  uint32_t stop_at = n;
+  while (p < n) {
+    uint32_t bits = 0;
+    if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
+    uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
+    uint32_t tok_len = 0, r = 0;
+    if (L == 0) {  // candidate position: one token
+      r = best_match(S, p, n, nruns, a, lane);
+      const uint32_t l = r >> 16;
+      tok_len = l >= a.m ? l : 1u;
+      L = 1;
+    }
+    // record token starts [p, p+L)
+    if (lane == 0) {
+      const uint32_t w = p >> 5, sh = p & 31u;
+      const uint32_t mask = L >= 32 ? 0xFFFFFFFFu : ((1u << L) - 1u);
+      atomicOr(&tbk[w], mask << sh);
+      if (sh + L > 32) atomicOr(&tbk[w + 1], mask >> (32 - sh));
+      if (tok_len > 1) d1[p] = (uint16_t)(0xFFFFu - (r & 0xFFFFu));  // d - 1
+    }
+    // does this stretch meet the successor's parse?
+    if (K > 1 && k + 1 < K && p + L > nb) {
+      const uint32_t pr = ld_volatile(&prog[k + 1]);
+      __threadfence_block();
+      const uint32_t lo = max(p, nb), hi = min(p + L, pr);
+      if (lo < hi) {
+        uint32_t x = hi;
+        for (uint32_t w = lo >> 5; w <= (hi - 1) >> 5; ++w) {
+          uint32_t b = ld_volatile(&tbn[w]);
+          const uint32_t wlo = w << 5;
+          if (wlo < lo) b &= 0xFFFFFFFFu << (lo - wlo);
+          if (hi - wlo < 32) b &= (1u << (hi - wlo)) - 1u;
+          if (b) {
+            x = wlo + (uint32_t)(__ffs(b) - 1);
+            break;
+          }
+        }
+        if (x < hi) {
+          stop_at = x;
+          if (lane == 0) {
+            __threadfence_block();
+            st_volatile(&prog[k], x + 1);
+          }
+          break;
+        }
       }
     }
-    carryT += __popc(tw);
-    carryM += __popc(mw);
+    p += tok_len ? tok_len : L;
+    if (lane == 0) {
+      __threadfence_block();
+      st_volatile(&prog[k], p);
+    }
   }
+  if (lane == 0) sync[k] = stop_at;
 }
 
-__global__ void __launch_bounds__(32 * kMaxWarps, 1) lzr_encode_kernel(const EncArgs a) {
+__device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
+  const uint32_t base = w << 5;
+  return n >= base + 32 ? 0xFFFFFFFFu : (n > base ? (1u << (n - base)) - 1u : 0u);
+}
+
+// threads per CTA at most: 10 groups of 1 or 2 warps, 9 of 3, 8 of 4
+template <int K>
+struct MaxThreads {
+  static constexpr int value = K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : 1024));
+};
+
+template <int K>
+__global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
   const uint32_t warp = threadIdx.x >> 5;
-  uint8_t* base = smem + (size_t)warp * a.L.per_warp;
+  const uint32_t g = warp / K, k = warp % K;  // group, warp within the group
+  const uint32_t bar_id = 1 + g, nthr = 32 * K;
+  uint8_t* base = smem + (size_t)g * a.L.per_group;
+  const uint32_t nw = a.L.bm_words;
   Smem S;
   S.data = base;
   S.sorted = reinterpret_cast<uint16_t*>(base + a.L.off_sorted);
   S.slot = reinterpret_cast<uint16_t*>(base + a.L.off_slot);
   uint32_t* bms = reinterpret_cast<uint32_t*>(base + a.L.off_bm);
-  const uint32_t nw = a.L.bm_words;
   S.cand = bms;
   S.cb = bms + nw;
-  S.tg = bms + 2 * nw;
-  S.flags = reinterpret_cast<uint8_t*>(bms + 4 * nw);
-  S.runs = reinterpret_cast<uint32_t*>(S.flags + align_up(a.C / 8, 4));
-  uint64_t* bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
+  S.tb = bms + 2 * nw;
+  S.runs = bms + (2 + K) * nw;
+  S.ctrl = S.runs + kMaxRuns;
+  S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
+  const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;
+  const uint32_t lt = lanemask_lt();
+  const uint32_t tid = k * 32 + lane;
 
-  if (lane == 0) {
-    mbar_init(bar, 1);
+  if (k == 0 && lane == 0) {
+    mbar_init(S.bar, 1);
     fence_mbar_init();
   }
-  __syncwarp();
   uint32_t phase = 0;
 
   for (;;) {
-    uint32_t c = 0;
-    if (lane == 0) c = atomicAdd(a.counter, 1u);
-    c = __shfl_sync(kFull, c, 0);
+    // ---- next chunk; all prior generic accesses to `data` before the TMA write
+    if (k == 0 && lane == 0) S.ctrl[kCtrlChunk] = atomicAdd(a.counter, 1u);
+    fence_proxy_async_smem();
+    group_sync(bar_id, nthr);
+    const uint32_t c = S.ctrl[kCtrlChunk];
     if (c >= a.N) break;
     const size_t lo = (size_t)c * a.C;
     const uint32_t n = (uint32_t)min((size_t)a.C, a.n_bytes - lo);
     const uint8_t* src = a.in + lo;
+    const uint32_t P = n >= a.m ? n - a.m + 1 : 0;  // positions that can start a match
+    uint8_t* out = a.slots + (size_t)c * (2 * a.C);  // workspace slot: d1 scratch, then the stream
+    uint16_t* d1 = reinterpret_cast<uint16_t*>(out);
 
-    // ---- a2: stage the chunk (TMA bulk for the 16-byte multiple, LDG for the tail)
-    fence_proxy_async_smem();  // prior generic accesses to `data` before the async write
-    __syncwarp();
+    // ---- a2: stage (TMA bulk for the 16-byte multiple, LDG for the tail); zero
+    //      the pre-filter, histogram and counters meanwhile
     const uint32_t n16 = n & ~15u;
-    if (lane == 0 && n16) {
-      mbar_arrive_expect_tx(bar, n16);
-      tma_bulk_g2s(S.data, src, n16, bar);
+    if (k == 0 && lane == 0 && n16) {
+      mbar_arrive_expect_tx(S.bar, n16);
+      tma_bulk_g2s(S.data, src, n16, S.bar);
     }
-    for (uint32_t i = n16 + lane; i < n; i += 32) S.data[i] = src[i];
-    for (uint32_t i = n + lane; i < align_up(n, 16) + 32; i += 32) S.data[i] = 0;
+    for (uint32_t i = n16 + tid; i < n; i += nthr) S.data[i] = src[i];
+    for (uint32_t i = n + tid; i < align_up(n, 16) + 32; i += nthr) S.data[i] = 0;
+    uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);    // B u16 counters
+    uint32_t* seen = reinterpret_cast<uint32_t*>(S.sorted);  // 2^fb-bit filter
+    for (uint32_t i = tid; i < B / 2; i += nthr) hist[i] = 0;
+    for (uint32_t i = tid; i < (1u << (fb - 5)); i += nthr) seen[i] = 0;
+    if (tid == 0) {
+      S.ctrl[kCtrlU] = 0;
+      S.ctrl[kCtrlRuns] = 0;
+    }
     if (n16) {
-      mbar_wait_parity(bar, phase);
+      mbar_wait_parity(S.bar, phase);
       phase ^= 1u;
     }
-    __syncwarp();
+    group_sync(bar_id, nthr);
 
-    const uint32_t P = n >= a.m ? n - a.m + 1 : 0;  // positions that can start a match
-    uint32_t nruns = 0;
-    bool raw = build_index(S, n, P, a, lane, nruns);
-
-    // ---- a3/a4: greedy walk.  Only matches are recorded (toggles, (d-1), (l-m));
-    // literal runs just advance p and the token count T; the flag byte of the
-    // current group of 8 tokens accumulates in a register.
-    uint32_t T = 0, Mt = 0;
-    uint32_t p = 0;
-    uint32_t gcur = 0, acc_f = 0;
-    while (!raw && p < n) {
-      uint32_t bits = 0;
-      if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
-      if (bits == 0) {  // 32 (or the rest) literals
-        const uint32_t L = min(32u, n - p);
-        T += L;
-        p += L;
-      } else {
-        const uint32_t f = (uint32_t)(__ffs(bits) - 1);  // literals before the candidate
-        T += f;
-        p += f;
-        const uint32_t r = best_match(S, p, n, nruns, a, lane);
-        const uint32_t l = r >> 16;
-        if (l >= a.m) {
-          if (lane == 0) {
-            atomicOr(&S.tg[(p + 1) >> 5], 1u << ((p + 1) & 31u));
-            atomicOr(&S.tg[(p + l) >> 5], 1u << ((p + l) & 31u));
-            S.slot[p] = (uint16_t)(0xFFFFu - (r & 0xFFFFu));  // d - 1
-            S.slot[p + 1] = (uint16_t)(l - a.m);
-          }
-          if ((T >> 3) != gcur) {
-            if (lane == 0 && acc_f) S.flags[gcur] = (uint8_t)acc_f;
-            gcur = T >> 3;
-            acc_f = 0;
-          }
-          acc_f |= 1u << (T & 7u);
-          Mt += 1;
-          p += l;
-        } else {
-          p += 1;
+    // ---- histogram of bucket sizes + "key hash seen before" count + run starts.
+    // Raw pre-filter (sound): a match of length l at s makes s..s+l-k positions
+    // with a same-key earlier occurrence, disjoint across matches; with
+    // X = sum(l-3) and T tokens, S = n - X + ceil(T/8) and T >= n - 3X (m >= 4)
+    // or n - 2(X + #matches) (m = 3), so S >= n whenever 11 * U <= n, U = number
+    // of positions whose key hash was seen before (>= that position count).
+    {
+      uint32_t u = 0;
+      for (uint32_t p0 = k * 32; p0 < P; p0 += nthr) {
+        const uint32_t p = p0 + lane;
+        bool dup = false, rs = false;
+        if (p < P) {
+          const uint32_t key = ld32u(S.data, p) & a.kmask;
+          const uint32_t h = khash(key, hb);
+          atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
+          const uint32_t gg = (key * 0x85EBCA6Bu) >> (32 - fb);
+          dup = atomicOr(&seen[gg >> 5], 1u << (gg & 31u)) & (1u << (gg & 31u));
+          rs = ((key ^ (key >> 8)) & (a.kmask >> 8)) == 0 && (p == 0 || S.data[p - 1] != S.data[p]);
         }
-        T += 1;
+        u += __popc(__ballot_sync(kFull, dup));
+        const uint32_t rb = __ballot_sync(kFull, rs);
+        if (rb) {
+          uint32_t b0 = 0;
+          if (lane == 0) b0 = atomicAdd(&S.ctrl[kCtrlRuns], (uint32_t)__popc(rb));
+          b0 = __shfl_sync(kFull, b0, 0);
+          const uint32_t idx = b0 + __popc(rb & lt);
+          if (rs && idx < kMaxRuns) S.runs[idx] = p;
+        }
       }
-      if (T + 2 * Mt + ((T + 7) >> 3) >= n) raw = true;  // not shorter than the chunk (R9)
+      if (lane == 0 && u) atomicAdd(&S.ctrl[kCtrlU], u);
     }
-    if (!raw && lane == 0 && acc_f) S.flags[gcur] = (uint8_t)acc_f;
-    __syncwarp();
-    uint32_t Sz = n;
-    if (!raw) {
-      Sz = T + 2 * Mt + ((T + 7) >> 3);
-      uint8_t* ob = reinterpret_cast<uint8_t*>(S.sorted);  // the index is dead now
-      encode_tokens(S, n, ob, lane);
-      __syncwarp();
-      uint8_t* out = a.slots + lo;
-      const uint32_t n16o = align_up(Sz, 16);
-      for (uint32_t i = lane * 16; i < n16o; i += 32 * 16)
-        *reinterpret_cast<uint4*>(out + i) = *reinterpret_cast<const uint4*>(ob + i);
+    group_sync(bar_id, nthr);
+    if (11u * S.ctrl[kCtrlU] <= n) {  // certainly raw
+      if (tid == 0) a.sizes[c] = n;
+      continue;
     }
-    if (lane == 0) a.sizes[c] = Sz;
-    __syncwarp();
+    const uint32_t nruns = S.ctrl[kCtrlRuns];
+
+    // ---- warp 0: exclusive scan of the B u16 counters (64 per round);
+    //      the other warps: zero the bitmaps, byte-change bitmap, walk state
+    const uint32_t kk = K == 1 ? 0 : k - 1, KK = K == 1 ? 1 : K - 1;  // helper warp index
+    if (k == 0) {
+      uint32_t carry = 0;
+      for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
+        const bool act = w0 + lane < B / 2;
+        const uint32_t wv = act ? hist[w0 + lane] : 0;
+        const uint32_t c0 = wv & 0xFFFFu, sum = c0 + (wv >> 16);
+        uint32_t incl = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t t = __shfl_up_sync(kFull, incl, o);
+          if ((int)lane >= o) incl += t;
+        }
+        const uint32_t excl = incl - sum + carry;
+        if (act) hist[w0 + lane] = (excl & 0xFFFFu) | ((excl + c0) << 16);
+        carry += __shfl_sync(kFull, incl, 31);
+      }
+    }
+    if (K == 1 || k != 0) {
+      for (uint32_t i = kk * 32 + lane; i < nw; i += KK * 32) S.cand[i] = 0;
+      for (uint32_t i = kk * 32 + lane; i < K * nw; i += KK * 32) S.tb[i] = 0;
+      for (uint32_t w = kk; w < nw; w += KK) {  // change bitmap
+        const uint32_t i = (w << 5) + lane;
+        const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
+        const uint32_t b = __ballot_sync(kFull, ch);
+        if (lane == 0) S.cb[w] = b;
+      }
+      if (kk == 0 && lane < K) {
+        S.ctrl[kCtrlProg + lane] = 0;      // prog
+        S.ctrl[kCtrlProg + K + lane] = n;  // sync
+      }
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- warp 0: stable scatter, 4 blocks of 32 positions per round so that the
+    //      MATCH.ANY latencies overlap; the other warps: run ends
+    if (k == 0) {
+      uint16_t* cur = S.slot;
+      for (uint32_t p0 = 0; p0 < P; p0 += 128) {
+        uint32_t h[4], peers[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t p = p0 + 32 * u + lane;
+          h[u] = p < P ? khash(ld32u(S.data, p) & a.kmask, hb) : 0xFFFFFFFFu;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t p = p0 + 32 * u + lane;
+          const bool act = p < P;
+          const uint32_t basev = act ? cur[h[u]] : 0;
+          if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)p;
+          __syncwarp();
+          if (act && lane == 31u - __clz(peers[u])) cur[h[u]] = (uint16_t)(basev + __popc(peers[u]));
+          __syncwarp();
+        }
+      }
+    }
+    if (K == 1 || k != 0) {
+      for (uint32_t j = kk * 32 + lane; j < min(nruns, kMaxRuns); j += KK * 32) {
+        const uint32_t st = S.runs[j];
+        S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
+      }
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- mark the first entry of every non-empty bucket (cur[h] = end of h)
+    for (uint32_t hh = tid; hh < B; hh += nthr) {
+      const uint32_t st = hh ? S.slot[hh - 1] : 0u;
+      if (S.slot[hh] > st) S.sorted[st] |= kFirst;
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- slot of each position and the candidate bitmap: the nearest same-key
+    //      earlier position is the nearest same-key entry below in the bucket
+    for (uint32_t sl = tid; sl < P; sl += nthr) {
+      const uint32_t e = S.sorted[sl];
+      const uint32_t q = e & kPos;
+      S.slot[q] = (uint16_t)sl;
+      if (!(e & kFirst)) {
+        const uint32_t kq = ld32u(S.data, q) & a.kmask;
+        bool has = false;
+        for (uint32_t s2 = sl - 1;; --s2) {
+          const uint32_t e2 = S.sorted[s2];
+          const uint32_t q2 = e2 & kPos;
+          if ((ld32u(S.data, q2) & a.kmask) == kq) {
+            has = q - q2 <= a.W;
+            break;
+          }
+          if (e2 & kFirst) break;
+        }
+        if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
+      }
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- a3/a4: the K speculative walk segments
+    {
+      const uint32_t start = (uint32_t)(((uint64_t)n * k) / K);
+      const uint32_t nb = (uint32_t)(((uint64_t)n * (k + 1)) / K);
+      if (start < n && (k == 0 || start > 0))
+        walk_segment<K>(S, d1, k, start, nb, n, P, nruns, a, lane);
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- final token-start bitmap = chain warp 0 -> warp 1 -> ... through the
+    //      meeting points (into the dead candidate bitmap); zero the
+    //      token-index match bitmap (dead byte-change bitmap)
+    for (uint32_t i = tid; i < nw; i += nthr) {
+      S.cand[i] = 0;
+      S.cb[i] = 0;
+    }
+    group_sync(bar_id, nthr);
+    {
+      uint32_t lo_k = 0, hi_k = 0;
+      bool in_chain = false;
+      uint32_t x = 0;
+      for (uint32_t w = 0; w < K; ++w) {
+        const uint32_t y = S.ctrl[kCtrlProg + K + w];
+        if (w == k) {
+          in_chain = true;
+          lo_k = x;
+          hi_k = y;
+        }
+        if (y >= n) break;
+        x = y;
+      }
+      if (in_chain && lo_k < hi_k) {
+        const uint32_t* tbk = S.tb + k * nw;
+        for (uint32_t w = (lo_k >> 5) + lane; w <= (hi_k - 1) >> 5; w += 32) {
+          uint32_t b = tbk[w];
+          const uint32_t wlo = w << 5;
+          if (wlo < lo_k) b &= 0xFFFFFFFFu << (lo_k - wlo);
+          if (hi_k - wlo < 32) b &= (1u << (hi_k - wlo)) - 1u;
+          if (b) atomicOr(&S.cand[w], b);
+        }
+      }
+      if (tid == 0) atomicOr(&S.cand[n >> 5], 1u << (n & 31u));  // sentinel: a token "starts" at n
+    }
+    group_sync(bar_id, nthr);
+
+    // ---- a5: totals.  A token at p is a match iff no token starts at p + 1.
+    const uint32_t nwords = (n + 31) >> 5;
+    const uint32_t w_lo = (nwords * k) / K, w_hi = (nwords * (k + 1)) / K;
+    {
+      uint32_t T = 0, M = 0;
+      for (uint32_t w = w_lo + lane; w < w_hi; w += 32) {
+        const uint32_t cw = S.cand[w];
+        const uint32_t t = cw & valid_mask(n, w);
+        const uint32_t mm = t & ~((cw >> 1) | (S.cand[w + 1] << 31));
+        T += __popc(t);
+        M += __popc(mm);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        T += __shfl_xor_sync(kFull, T, o);
+        M += __shfl_xor_sync(kFull, M, o);
+      }
+      if (lane == 0) {
+        S.ctrl[kCtrlProg + 2 * K + k] = T;
+        S.ctrl[kCtrlProg + 3 * K + k] = M;
+      }
+    }
+    group_sync(bar_id, nthr);
+    uint32_t Ttot = 0, Mtot = 0, Tb = 0, Mb = 0;
+    for (uint32_t w = 0; w < K; ++w) {
+      const uint32_t t = S.ctrl[kCtrlProg + 2 * K + w], m = S.ctrl[kCtrlProg + 3 * K + w];
+      if (w < k) {
+        Tb += t;
+        Mb += m;
+      }
+      Ttot += t;
+      Mtot += m;
+    }
+    const uint32_t Sz = Ttot + 2 * Mtot + ((Ttot + 7) >> 3);
+    if (Sz >= n) {  // not shorter than the chunk: stored raw (R9)
+      if (tid == 0) a.sizes[c] = n;
+      continue;
+    }
+
+    // ---- pass 0: match bit per token index (source of the flag bytes);
+    //      pass 1: every token's bytes.  The warp's words in rounds of 32:
+    //      lane-parallel counts + scan give each word's token/match bases.
+    uint8_t* ob = reinterpret_cast<uint8_t*>(S.sorted);  // the index is dead now
+    for (int pass = 0; pass < 2; ++pass) {
+      uint32_t tb_run = Tb, mb_run = Mb;
+      for (uint32_t w0 = w_lo; w0 < w_hi; w0 += 32) {
+        const uint32_t w = w0 + lane;
+        uint32_t t = 0, mm = 0;
+        if (w < w_hi) {
+          const uint32_t cw = S.cand[w];
+          t = cw & valid_mask(n, w);
+          mm = t & ~((cw >> 1) | (S.cand[w + 1] << 31));
+        }
+        const uint32_t pt = __popc(t), pm = __popc(mm);
+        uint32_t ti = pt, mi = pm;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t a1 = __shfl_up_sync(kFull, ti, o), b1 = __shfl_up_sync(kFull, mi, o);
+          if ((int)lane >= o) {
+            ti += a1;
+            mi += b1;
+          }
+        }
+        const uint32_t tbase = tb_run + ti - pt, mbase = mb_run + mi - pm;
+        tb_run += __shfl_sync(kFull, ti, 31);
+        mb_run += __shfl_sync(kFull, mi, 31);
+        if (pass == 0) {
+          uint32_t rem = mm;  // this lane's word: token indices of its matches
+          while (rem) {
+            const uint32_t bit = (uint32_t)(__ffs(rem) - 1);
+            rem &= rem - 1;
+            const uint32_t j = tbase + __popc(t & ((1u << bit) - 1u));
+            atomicOr(&S.cb[j >> 5], 1u << (j & 31u));
+          }
+        } else {
+          const uint32_t nwr = min(32u, w_hi - w0);
+          for (uint32_t i = 0; i < nwr; ++i) {
+            const uint32_t tw = __shfl_sync(kFull, t, i), mw = __shfl_sync(kFull, mm, i);
+            const uint32_t tbw = __shfl_sync(kFull, tbase, i), mbw = __shfl_sync(kFull, mbase, i);
+            if ((tw >> lane) & 1u) {
+              const uint32_t p = ((w0 + i) << 5) + lane;
+              const uint32_t j = tbw + __popc(tw & lt);
+              const uint32_t mbef = mbw + __popc(mw & lt);
+              const uint32_t pos = j + 2 * mbef + (j >> 3) + 1;
+              if ((j & 7u) == 0) ob[pos - 1] = (uint8_t)(S.cb[j >> 5] >> (j & 24u));
+              if ((mw >> lane) & 1u) {
+                // length = distance to the next token start (sentinel at n)
+                uint32_t ww = (p + 1) >> 5;
+                uint32_t b = S.cand[ww] & (0xFFFFFFFFu << ((p + 1) & 31u));
+                while (!b) b = S.cand[++ww];
+                const uint32_t l = (ww << 5) + (uint32_t)(__ffs(b) - 1) - p;
+                const uint32_t dm1 = d1[p];
+                ob[pos] = (uint8_t)(dm1 & 0xFF);
+                ob[pos + 1] = (uint8_t)(dm1 >> 8);
+                ob[pos + 2] = (uint8_t)(l - a.m);
+              } else {
+                ob[pos] = S.data[p];
+              }
+            }
+          }
+        }
+      }
+      group_sync(bar_id, nthr);
+    }
+
+    // ---- copy the staged stream to the chunk's workspace slot (16-byte stores;
+    //      every d1 read happened before the last group barrier)
+    const uint32_t n16o = align_up(Sz, 16);
+    for (uint32_t i = tid * 16; i < n16o; i += nthr * 16)
+      *reinterpret_cast<uint4*>(out + i) = *reinterpret_cast<const uint4*>(ob + i);
+    if (tid == 0) a.sizes[c] = Sz;
   }
+}
+
+template <int K>
+cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
+  int groups = smem_optin / (int)a.L.per_group;
+  const int max_groups = MaxThreads<K>::value / (32 * K);
+  if (groups > max_groups) groups = max_groups;
+  if (groups > 15) groups = 15;  // named barriers 1..15
+  if (groups < 1) return cudaErrorInvalidConfiguration;
+  const size_t smem = (size_t)groups * a.L.per_group;
+  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (err != cudaSuccess) return err;
+  const uint32_t need = (a.N + groups - 1) / groups;
+  const uint32_t grid = need < (uint32_t)sm_count ? need : (uint32_t)sm_count;
+  lzr_encode_kernel<K><<<grid, groups * 32 * K, smem, s>>>(a);
+  if (launches) ++*launches;
+  return cudaGetLastError();
 }
 
 }  // namespace
 
 cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s,
                           int* launches) {
-  int warps = smem_optin / (int)a.L.per_warp;
-  if (warps > kMaxWarps) warps = kMaxWarps;
-  if (warps < 1) return cudaErrorInvalidConfiguration;
-  const size_t smem = (size_t)warps * a.L.per_warp;
-  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (err != cudaSuccess) return err;
-  const uint32_t need = (a.N + warps - 1) / warps;
-  const uint32_t grid = need < (uint32_t)sm_count ? need : (uint32_t)sm_count;
-  lzr_encode_kernel<<<grid, warps * 32, smem, s>>>(a);
-  if (launches) ++*launches;
-  return cudaGetLastError();
+  switch (a.L.K) {
+    case 1: return launch_k<1>(a, sm_count, smem_optin, s, launches);
+    case 2: return launch_k<2>(a, sm_count, smem_optin, s, launches);
+    case 3: return launch_k<3>(a, sm_count, smem_optin, s, launches);
+    case 4: return launch_k<4>(a, sm_count, smem_optin, s, launches);
+    default: return cudaErrorInvalidConfiguration;
+  }
 }
 
 }  // namespace lzr

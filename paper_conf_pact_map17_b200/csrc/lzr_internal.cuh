@@ -69,9 +69,9 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
   }
 }
 
-// ---- encode kernel shared-memory layout (one region per warp = per chunk) ---
+// ---- encode kernel shared-memory layout (one region per group of K warps) ---
 struct EncLayout {
-  uint32_t off_sorted, off_slot, off_bm, off_mbar, per_warp, hbits, bm_words, fbits;
+  uint32_t K, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, fbits;
 };
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
@@ -80,8 +80,9 @@ __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
   return hb;
 }
 
-__host__ __device__ inline EncLayout enc_layout(uint32_t C) {
+__host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K) {
   EncLayout L;
+  L.K = K;
   L.hbits = enc_hash_bits(C);
   L.fbits = 5;  // raw pre-filter: 2^fbits bits inside the 2C-byte index region, <= 2^15
   while ((2u << L.fbits) <= 16 * C && L.fbits < 15) ++L.fbits;
@@ -90,16 +91,14 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C) {
   L.off_sorted = o;
   o = align_up(o + 2 * C, 16);  // u16 positions grouped by hash bucket, ascending
   L.off_slot = o;
-  o = align_up(o + 2 * (C > B ? C : B), 16);  // u16 slot of each position (histogram before)
+  o = align_up(o + 2 * (C > B ? C : B), 16);  // u16 histogram -> cursors -> slot of each position
   L.off_bm = o;
   L.bm_words = (C + 31) / 32 + 1;  // +1: two-word funnel reads at the last position
-  // four bitmaps (candidate, byte-change, token start, match), group flag bytes
-  // (C/8) and the run list (32 entries); sized so that 10 warps (chunks) fit one
-  // SM at C = 4096
-  o = align_up(o + 4 * 4 * L.bm_words + align_up(C / 8, 4) + 4 * 32, 16);
+  // bitmaps: candidate, byte-change, K token-start; run list (32); ctrl (4 + 4K)
+  o = align_up(o + 4 * ((2 + K) * L.bm_words + 32 + 4 + 4 * K), 16);
   L.off_mbar = o;
   o += 16;
-  L.per_warp = align_up(o, 16);
+  L.per_group = align_up(o, 16);
   return L;
 }
 
@@ -110,7 +109,7 @@ struct EncArgs {
   uint32_t C, W, m, M;
   uint32_t kbytes, kmask;  // candidate key = first min(m,4) bytes
   EncLayout L;
-  uint8_t* slots;  // workspace: chunk i stream at slots + i*C
+  uint8_t* slots;  // workspace: chunk i at slots + i*2C (u16 (d-1) scratch, then its stream)
   uint32_t* sizes;
   uint32_t* counter;  // work distribution, zeroed before launch
 };
@@ -127,6 +126,7 @@ cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaSt
 cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, uint64_t* offsets,
                         uint64_t* total, void* ws, cudaStream_t s, int* launches);
 cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const uint8_t* slots,
+                           size_t slot_stride,
                            const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,
                            int sm_count, cudaStream_t s, int* launches);
 cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,

@@ -131,6 +131,7 @@ __device__ __forceinline__ void warp_copy(uint8_t* dst, const uint8_t* src, uint
 __global__ void __launch_bounds__(256) lzr_compact_kernel(const uint8_t* __restrict__ in,
                                                           size_t n_bytes, uint32_t C,
                                                           const uint8_t* __restrict__ slots,
+                                                          size_t slot_stride,
                                                           const uint32_t* __restrict__ sizes,
                                                           const uint64_t* __restrict__ offsets,
                                                           uint8_t* __restrict__ out, size_t N) {
@@ -141,7 +142,7 @@ __global__ void __launch_bounds__(256) lzr_compact_kernel(const uint8_t* __restr
     const size_t lo = i * C;
     const uint32_t ni = (uint32_t)min((size_t)C, n_bytes - lo);
     const uint32_t S = sizes[i];
-    const uint8_t* src = (S == ni) ? in + lo : slots + lo;  // raw chunk: copy the input (R9)
+    const uint8_t* src = (S == ni) ? in + lo : slots + i * slot_stride;  // raw: the input (R9)
     warp_copy(out + offsets[i], src, S, lane);
   }
 }
@@ -166,14 +167,15 @@ cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, uint64_t
 }
 
 cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const uint8_t* slots,
-                           const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,
+                           size_t slot_stride, const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,
                            int sm_count, cudaStream_t s, int* launches) {
   const size_t N = (n_bytes + C - 1) / C;
   if (N == 0) return cudaSuccess;
   size_t blocks = (N + 7) / 8;
   const size_t cap = (size_t)sm_count * 8;
   if (blocks > cap) blocks = cap;
-  lzr_compact_kernel<<<(unsigned)blocks, 256, 0, s>>>(in, n_bytes, C, slots, sizes, offsets, out, N);
+  lzr_compact_kernel<<<(unsigned)blocks, 256, 0, s>>>(in, n_bytes, C, slots, slot_stride, sizes,
+                                                     offsets, out, N);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
