@@ -21,7 +21,8 @@ __all__ = [
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "liblzr.so")
+# LZR_LIBRARY may point at an instrumented build of the same sources (profiling)
+LIB_PATH = os.environ.get("LZR_LIBRARY") or os.path.join(_PKG, "liblzr.so")
 
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CAPACITY, ERR_CUDA, ERR_CORRUPT = 0, -1, -2, -3, -4, -5
 

@@ -35,6 +35,13 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps())
 
 
+def build_timing() -> str:
+    """Instrumented variant (per-phase cycle counters, tools/phase_times.py)."""
+    out = os.path.join(PKG, "liblzr_timing.so")
+    subprocess.check_call(["nvcc", *NVCC_FLAGS, "-DLZR_PHASE_TIMING", "-o", out, *sources()])
+    return out
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if force or stale():
         cmd = ["nvcc", *NVCC_FLAGS, *(["-Xptxas", "-v"] if verbose else []),
@@ -46,5 +53,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 if __name__ == "__main__":
     import sys
-    build(force="-f" in sys.argv, verbose="-v" in sys.argv)
-    print(LIB)
+    if "--timing" in sys.argv:
+        print(build_timing())
+    else:
+        build(force="-f" in sys.argv, verbose="-v" in sys.argv)
+        print(LIB)

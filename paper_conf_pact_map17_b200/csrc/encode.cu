@@ -46,13 +46,39 @@ constexpr uint32_t kMaxRuns = 32;  // runs of one byte value of length >= k, per
 // ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K], T[K], M[K]
 constexpr int kCtrlChunk = 0, kCtrlU = 1, kCtrlRuns = 2, kCtrlProg = 4;
 
-__device__ __forceinline__ uint32_t khash(uint32_t key, uint32_t hbits) {
-  return (key * 0x9E3779B1u) >> (32 - hbits);
+// Bucket of a key.  With >= 1024 buckets, keys that are one repeated byte get
+// private buckets 0..255 (their buckets can hold thousands of positions, e.g.
+// zero runs, and a colliding key would scan them all); other keys hash into
+// the remaining B - 256.
+__device__ __forceinline__ uint32_t khash(uint32_t key, uint32_t hbits, uint32_t kmask) {
+  const uint32_t h = (key * 0x9E3779B1u) >> (32 - hbits);
+  if (hbits < 10) return h;
+  if (((key ^ (key >> 8)) & (kmask >> 8)) == 0) return key & 0xFFu;
+  return 256u + ((h * ((1u << hbits) - 256u)) >> hbits);
 }
 
 __device__ __forceinline__ void group_sync(uint32_t id, uint32_t nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
+
+#ifdef LZR_PHASE_TIMING
+// debug build only: per phase and warp-in-group, cycles working / waiting at
+// the group barrier that closes the phase
+__device__ unsigned long long g_phase[16][4][2];
+#define GSYNC(ph)                                                            \
+  do {                                                                       \
+    const long long t_arr = clock64();                                       \
+    group_sync(bar_id, nthr);                                                \
+    const long long t_lv = clock64();                                        \
+    if (lane == 0) {                                                         \
+      atomicAdd(&g_phase[ph][k & 3][0], (unsigned long long)(t_arr - t_ph)); \
+      atomicAdd(&g_phase[ph][k & 3][1], (unsigned long long)(t_lv - t_arr)); \
+    }                                                                        \
+    t_ph = t_lv;                                                             \
+  } while (0)
+#else
+#define GSYNC(ph) group_sync(bar_id, nthr)
+#endif
 
 __device__ __forceinline__ uint32_t ld_volatile(const uint32_t* p) {
   return *reinterpret_cast<const volatile uint32_t*>(p);
@@ -220,6 +246,35 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
     uint32_t lim = 32;
     if (m_first) lim = (uint32_t)__ffs(m_first);
     if (m_stop) lim = min(lim, (uint32_t)(__ffs(m_stop) - 1));
+    if (lim <= 8 && blen == 0 && !rp) {
+      // few candidates (the whole list): G lanes per candidate, 4 bytes per
+      // lane per step, first mismatch by ballot -- no per-lane compare loop
+      const uint32_t G = lim <= 4 ? 8u : 4u;
+      const uint32_t ci = lane / G, j = lane % G;
+      const uint32_t qc = __shfl_sync(kFull, q, ci & 31u);
+      const bool act = ci < lim;
+      const uint32_t gmask = ((1u << G) - 1u) << (ci * G);
+      uint32_t l = 0;
+      bool done = !act;
+      for (uint32_t off0 = 0;; off0 += 4 * G) {
+        const uint32_t off = off0 + 4 * j;
+        uint32_t x = 0;
+        if (!done) x = ld32u(data, p + off) ^ ld32u(data, qc + off);
+        const bool stop = !done && (x != 0 || off + 4 >= cap);
+        const uint32_t sm = __ballot_sync(kFull, stop) & gmask;
+        const uint32_t src = sm ? (uint32_t)(__ffs(sm) - 1) : lane;  // first stop in my group
+        const uint32_t xf = __shfl_sync(kFull, x, src);
+        if (!done && sm) {
+          l = off0 + 4 * (src - ci * G) + (xf ? ((uint32_t)(__ffs(xf) - 1) >> 3) : 4u);
+          if (l > cap) l = cap;
+          done = true;
+        }
+        if (__all_sync(kFull, done)) break;
+      }
+      uint32_t pk = 0;
+      if (act && j == 0 && l >= a.m) pk = (l << 16) | (0xFFFFu - (p - qc - 1));
+      return __reduce_max_sync(kFull, pk);
+    }
     uint32_t pk = 0;
     if (lane < lim && (blen == 0 || data[q + blen] == data[p + blen])) {
       uint32_t l;
@@ -316,6 +371,15 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
   if (lane == 0) sync[k] = stop_at;
 }
 
+__device__ __forceinline__ uint32_t walk_bound(uint32_t n, uint32_t k, uint32_t K) {
+  if (k == 0) return 0;
+  if (k >= K) return n;
+  // density 1 + 0.5 x  =>  bound = (sqrt(1 + 1.25 k/K) - 1) / 0.5
+  const float f = 2.0f * (sqrtf(1.0f + 1.25f * (float)k / (float)K) - 1.0f);
+  const uint32_t b = (uint32_t)(f * (float)n);
+  return b < n ? b : n;
+}
+
 __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
   const uint32_t base = w << 5;
   return n >= base + 32 ? 0xFFFFFFFFu : (n > base ? (1u << (n - base)) - 1u : 0u);
@@ -356,12 +420,20 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     fence_mbar_init();
   }
   uint32_t phase = 0;
+  uint32_t next_c = 0;  // leader: prefetched next chunk index (atomic latency hidden)
+  if (k == 0 && lane == 0) next_c = atomicAdd(a.counter, 1u);
+#ifdef LZR_PHASE_TIMING
+  long long t_ph = clock64();
+#endif
 
   for (;;) {
     // ---- next chunk; all prior generic accesses to `data` before the TMA write
-    if (k == 0 && lane == 0) S.ctrl[kCtrlChunk] = atomicAdd(a.counter, 1u);
+    if (k == 0 && lane == 0) {
+      S.ctrl[kCtrlChunk] = next_c;
+      next_c = atomicAdd(a.counter, 1u);
+    }
     fence_proxy_async_smem();
-    group_sync(bar_id, nthr);
+    GSYNC(0);
     const uint32_t c = S.ctrl[kCtrlChunk];
     if (c >= a.N) break;
     const size_t lo = (size_t)c * a.C;
@@ -392,7 +464,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       mbar_wait_parity(S.bar, phase);
       phase ^= 1u;
     }
-    group_sync(bar_id, nthr);
+    GSYNC(1);
 
     // ---- histogram of bucket sizes + "key hash seen before" count + run starts.
     // Raw pre-filter (sound): a match of length l at s makes s..s+l-k positions
@@ -405,14 +477,26 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       for (uint32_t p0 = k * 32; p0 < P; p0 += nthr) {
         const uint32_t p = p0 + lane;
         bool dup = false, rs = false;
-        if (p < P) {
-          const uint32_t key = ld32u(S.data, p) & a.kmask;
-          const uint32_t h = khash(key, hb);
+        const uint32_t key = p < P ? ld32u(S.data, p) & a.kmask : 0u;
+        // 32 equal keys (a run): one atomic each instead of 32 on one address
+        const uint32_t key0 = __shfl_sync(kFull, key, 0);
+        const bool uni = __all_sync(kFull, p < P && key == key0);
+        const uint32_t h = khash(key, hb, a.kmask);
+        const uint32_t gg = (key * 0x85EBCA6Bu) >> (32 - fb);
+        if (uni) {
+          uint32_t old = 0;
+          if (lane == 0) {
+            atomicAdd(&hist[h >> 1], 32u << ((h & 1u) << 4));
+            old = atomicOr(&seen[gg >> 5], 1u << (gg & 31u));
+          }
+          old = __shfl_sync(kFull, old, 0);
+          dup = lane ? true : (old & (1u << (gg & 31u))) != 0;
+        } else if (p < P) {
           atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
-          const uint32_t gg = (key * 0x85EBCA6Bu) >> (32 - fb);
           dup = atomicOr(&seen[gg >> 5], 1u << (gg & 31u)) & (1u << (gg & 31u));
-          rs = ((key ^ (key >> 8)) & (a.kmask >> 8)) == 0 && (p == 0 || S.data[p - 1] != S.data[p]);
         }
+        if (p < P)
+          rs = ((key ^ (key >> 8)) & (a.kmask >> 8)) == 0 && (p == 0 || S.data[p - 1] != S.data[p]);
         u += __popc(__ballot_sync(kFull, dup));
         const uint32_t rb = __ballot_sync(kFull, rs);
         if (rb) {
@@ -425,7 +509,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       }
       if (lane == 0 && u) atomicAdd(&S.ctrl[kCtrlU], u);
     }
-    group_sync(bar_id, nthr);
+    GSYNC(2);
     if (11u * S.ctrl[kCtrlU] <= n) {  // certainly raw
       if (tid == 0) a.sizes[c] = n;
       continue;
@@ -466,7 +550,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         S.ctrl[kCtrlProg + K + lane] = n;  // sync
       }
     }
-    group_sync(bar_id, nthr);
+    GSYNC(3);
 
     // ---- warp 0: stable scatter, 4 blocks of 32 positions per round so that the
     //      MATCH.ANY latencies overlap; the other warps: run ends
@@ -477,7 +561,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const uint32_t p = p0 + 32 * u + lane;
-          h[u] = p < P ? khash(ld32u(S.data, p) & a.kmask, hb) : 0xFFFFFFFFu;
+          h[u] = p < P ? khash(ld32u(S.data, p) & a.kmask, hb, a.kmask) : 0xFFFFFFFFu;
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
@@ -499,14 +583,14 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
       }
     }
-    group_sync(bar_id, nthr);
+    GSYNC(4);
 
     // ---- mark the first entry of every non-empty bucket (cur[h] = end of h)
     for (uint32_t hh = tid; hh < B; hh += nthr) {
       const uint32_t st = hh ? S.slot[hh - 1] : 0u;
       if (S.slot[hh] > st) S.sorted[st] |= kFirst;
     }
-    group_sync(bar_id, nthr);
+    GSYNC(5);
 
     // ---- slot of each position and the candidate bitmap: the nearest same-key
     //      earlier position is the nearest same-key entry below in the bucket
@@ -529,17 +613,25 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
       }
     }
-    group_sync(bar_id, nthr);
+    GSYNC(6);
 
     // ---- a3/a4: the K speculative walk segments
     {
-      const uint32_t start = (uint32_t)(((uint64_t)n * k) / K);
-      const uint32_t nb = (uint32_t)(((uint64_t)n * (k + 1)) / K);
+      // later positions have more candidates: segment bounds balance a work
+      // density growing ~linearly with the position (walk_bound)
+      const uint32_t start = walk_bound(n, k, K), nb = walk_bound(n, k + 1, K);
       if (start < n && (k == 0 || start > 0))
         walk_segment<K>(S, d1, k, start, nb, n, P, nruns, a, lane);
     }
-    group_sync(bar_id, nthr);
+    GSYNC(7);
 
+    // ---- (d-1) of the recorded matches: global scratch -> the dead slot array
+    //      (one parallel 16-byte copy instead of per-token global latencies)
+    {
+      const uint4* srcv = reinterpret_cast<const uint4*>(d1);
+      uint4* dstv = reinterpret_cast<uint4*>(S.slot);
+      for (uint32_t i = tid; i < (n + 7) / 8; i += nthr) dstv[i] = __ldcg(srcv + i);
+    }
     // ---- final token-start bitmap = chain warp 0 -> warp 1 -> ... through the
     //      meeting points (into the dead candidate bitmap); zero the
     //      token-index match bitmap (dead byte-change bitmap)
@@ -547,7 +639,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       S.cand[i] = 0;
       S.cb[i] = 0;
     }
-    group_sync(bar_id, nthr);
+    GSYNC(8);
     {
       uint32_t lo_k = 0, hi_k = 0;
       bool in_chain = false;
@@ -574,7 +666,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       }
       if (tid == 0) atomicOr(&S.cand[n >> 5], 1u << (n & 31u));  // sentinel: a token "starts" at n
     }
-    group_sync(bar_id, nthr);
+    GSYNC(9);
 
     // ---- a5: totals.  A token at p is a match iff no token starts at p + 1.
     const uint32_t nwords = (n + 31) >> 5;
@@ -598,7 +690,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         S.ctrl[kCtrlProg + 3 * K + k] = M;
       }
     }
-    group_sync(bar_id, nthr);
+    GSYNC(10);
     uint32_t Ttot = 0, Mtot = 0, Tb = 0, Mb = 0;
     for (uint32_t w = 0; w < K; ++w) {
       const uint32_t t = S.ctrl[kCtrlProg + 2 * K + w], m = S.ctrl[kCtrlProg + 3 * K + w];
@@ -667,7 +759,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
                 uint32_t b = S.cand[ww] & (0xFFFFFFFFu << ((p + 1) & 31u));
                 while (!b) b = S.cand[++ww];
                 const uint32_t l = (ww << 5) + (uint32_t)(__ffs(b) - 1) - p;
-                const uint32_t dm1 = d1[p];
+                const uint32_t dm1 = S.slot[p];
                 ob[pos] = (uint8_t)(dm1 & 0xFF);
                 ob[pos + 1] = (uint8_t)(dm1 >> 8);
                 ob[pos + 2] = (uint8_t)(l - a.m);
@@ -678,7 +770,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
           }
         }
       }
-      group_sync(bar_id, nthr);
+      GSYNC(11);
     }
 
     // ---- copy the staged stream to the chunk's workspace slot (16-byte stores;
@@ -709,6 +801,14 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
 }
 
 }  // namespace
+
+#ifdef LZR_PHASE_TIMING
+extern "C" int lzr_debug_phase_times(unsigned long long* out) {
+  if (cudaMemcpyFromSymbol(out, g_phase, sizeof(g_phase)) != cudaSuccess) return -4;
+  static unsigned long long zero[16][4][2];
+  return cudaMemcpyToSymbol(g_phase, zero, sizeof(g_phase)) == cudaSuccess ? 0 : -4;
+}
+#endif
 
 cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s,
                           int* launches) {
