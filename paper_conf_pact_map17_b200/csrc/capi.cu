@@ -61,9 +61,16 @@ WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
   WsLayout w;
   const size_t C = p->chunk_size;
   const size_t N = (n_bytes + C - 1) / C;
+  DevInfo di;
+  const size_t sms = dev_info(&di) == cudaSuccess ? (size_t)di.sm_count : 1024;
+  // resident chunk groups: grid (<= SMs) x groups per CTA (<= 16); the launch
+  // uses at most ceil(N / groups) CTAs, i.e. at most N + 15 groups
+  size_t groups = sms * kMaxGroupsPerSm;
+  if (groups > N + kMaxGroupsPerSm) groups = N + kMaxGroupsPerSm;
   w.ctrl_off = 0;
   w.slots_off = 256;
-  w.scan_off = w.slots_off + align_up_z(N * 2 * C, 256);  // per chunk: (d-1) scratch, then stream
+  w.scratch_off = w.slots_off + align_up_z(N * C, 256);
+  w.scan_off = w.scratch_off + align_up_z(groups * 2 * C, 256);
   w.total = w.scan_off + scan_ws_bytes(N);
   return w;
 }
@@ -146,6 +153,7 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   if (p->chunk_size > 32768 || (int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;
   uint8_t* ws = (uint8_t*)d_workspace;
   a.slots = ws + w.slots_off;
+  a.scratch = ws + w.scratch_off;
   a.sizes = d_sizes;
   a.counter = (uint32_t*)(ws + w.ctrl_off);
   cudaStream_t s = (cudaStream_t)stream;
@@ -180,7 +188,7 @@ int lzr_compress_compact(const void* d_in, size_t n_bytes, const lzr_params* p, 
   if (launch_scan(d_sizes, N, 0, d_offsets, d_total, ws + w.scan_off, s, &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
   if (launch_compact((const uint8_t*)d_in, n_bytes, p->chunk_size, ws + w.slots_off,
-                     2 * (size_t)p->chunk_size, d_sizes,
+                     (size_t)p->chunk_size, d_sizes,
                      d_offsets, (uint8_t*)d_out, di.sm_count, s, &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;

@@ -299,9 +299,9 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 
 // ---- a4: one speculative walk segment ----------------------------------------
 // Warp k parses greedily from `start`.  Token starts go into its bitmap tbk
-// (lane 0, atomics), (d-1) into d1[s] at each match start s (global scratch in
-// the chunk's workspace slot; identical from every warp that records a token
-// at s, since the best match at s does not depend on the parse).  prog[k]: every token start of warp k below prog[k] is
+// (lane 0, atomics), (d-1) into d1[s] at each match start s (the group's global
+// scratch; identical from every warp that records a token at s, since the best
+// match at s does not depend on the parse).  prog[k]: every token start of warp k below prog[k] is
 // recorded.  A warp with a successor stops at the first of its token starts x
 // that the successor has recorded (x < prog[k+1]); sync[k] = x, or n if it ran
 // to the end.
@@ -414,6 +414,10 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
   const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;
   const uint32_t lt = lanemask_lt();
   const uint32_t tid = k * 32 + lane;
+  // (d-1) of recorded matches: a per-group global scratch reused chunk after
+  // chunk (stays in L2); read back only at the final match starts
+  uint16_t* d1 = reinterpret_cast<uint16_t*>(
+      a.scratch + ((size_t)blockIdx.x * (blockDim.x / (32 * K)) + g) * (2 * (size_t)a.C));
 
   if (k == 0 && lane == 0) {
     mbar_init(S.bar, 1);
@@ -440,8 +444,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     const uint32_t n = (uint32_t)min((size_t)a.C, a.n_bytes - lo);
     const uint8_t* src = a.in + lo;
     const uint32_t P = n >= a.m ? n - a.m + 1 : 0;  // positions that can start a match
-    uint8_t* out = a.slots + (size_t)c * (2 * a.C);  // workspace slot: d1 scratch, then the stream
-    uint16_t* d1 = reinterpret_cast<uint16_t*>(out);
+    uint8_t* out = a.slots + (size_t)c * a.C;  // the chunk's workspace slot (its stream)
 
     // ---- a2: stage (TMA bulk for the 16-byte multiple, LDG for the tail); zero
     //      the pre-filter, histogram and counters meanwhile
@@ -625,13 +628,6 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     }
     GSYNC(7);
 
-    // ---- (d-1) of the recorded matches: global scratch -> the dead slot array
-    //      (one parallel 16-byte copy instead of per-token global latencies)
-    {
-      const uint4* srcv = reinterpret_cast<const uint4*>(d1);
-      uint4* dstv = reinterpret_cast<uint4*>(S.slot);
-      for (uint32_t i = tid; i < (n + 7) / 8; i += nthr) dstv[i] = __ldcg(srcv + i);
-    }
     // ---- final token-start bitmap = chain warp 0 -> warp 1 -> ... through the
     //      meeting points (into the dead candidate bitmap); zero the
     //      token-index match bitmap (dead byte-change bitmap)
@@ -741,6 +737,8 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
             rem &= rem - 1;
             const uint32_t j = tbase + __popc(t & ((1u << bit) - 1u));
             atomicOr(&S.cb[j >> 5], 1u << (j & 31u));
+            const uint32_t pm = (w << 5) + bit;
+            S.slot[pm] = __ldcg(d1 + pm);  // the slot array is dead after the walk
           }
         } else {
           const uint32_t nwr = min(32u, w_hi - w0);

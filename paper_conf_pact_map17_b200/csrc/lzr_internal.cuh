@@ -109,15 +109,17 @@ struct EncArgs {
   uint32_t C, W, m, M;
   uint32_t kbytes, kmask;  // candidate key = first min(m,4) bytes
   EncLayout L;
-  uint8_t* slots;  // workspace: chunk i at slots + i*2C (u16 (d-1) scratch, then its stream)
+  uint8_t* slots;    // workspace: chunk i's stream at slots + i*C
+  uint8_t* scratch;  // workspace: 2C bytes per resident group (u16 (d-1) per position)
   uint32_t* sizes;
   uint32_t* counter;  // work distribution, zeroed before launch
 };
 
 // ---- workspace layout ---------------------------------------------------------
 struct WsLayout {
-  size_t ctrl_off, slots_off, scan_off, total;
+  size_t ctrl_off, slots_off, scratch_off, scan_off, total;
 };
+constexpr uint32_t kMaxGroupsPerSm = 16;  // scratch bound: groups per CTA (one CTA per SM)
 size_t scan_ws_bytes(size_t n);
 WsLayout ws_layout(size_t n_bytes, const lzr_params* p);
 
