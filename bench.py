@@ -220,7 +220,9 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    # under torchrun the sharded path (NCCL all-gather of sizes) runs even at N = 1
+    sharded = "WORLD_SIZE" in os.environ and "MASTER_ADDR" in os.environ
+    if sharded:
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
     p = lzr.Params(chunk_size=C)
@@ -229,7 +231,7 @@ def main():
     stream = torch.cuda.current_stream(dev)
 
     # ---- inputs, generated on each GPU (global chunk indices of this shard)
-    if world > 1:
+    if sharded:
         sc = ShardedCompressor(n_glob, p, None, dev)
         assert sc.n_local == n_rank
         first = sc.lo
@@ -238,14 +240,14 @@ def main():
     x = torch.empty(n_rank, dtype=torch.uint8, device=dev)
     synth.fill_device(x, C, a.cls, first_chunk=first)
     ws = lzr.Workspace(n_rank, p, dev)
-    if world > 1:
+    if sharded:
         sc.ops.ws = ws
         sc.ops.bind_sizes(sc.sizes_pad)
 
     launches = [0]
 
     def step(ev_enc=None):
-        if world > 1:
+        if sharded:
             if ev_enc is not None:
                 ev_enc[0].record(stream)
             lzr.compress_encode(x, p, ws)
@@ -270,7 +272,7 @@ def main():
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
-    if world > 1:
+    if sharded:
         dist.barrier()
     enc_events = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                   for _ in range(a.steps)]
@@ -278,18 +280,18 @@ def main():
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
-        if world > 1:
+        if sharded:
             dist.barrier()
         t_start.record(stream)
         for k in range(a.steps):
             step(enc_events[k])
         t_end.record(stream)
         torch.cuda.synchronize()
-        if world > 1:
+        if sharded:
             dist.barrier()
     ms = t_start.elapsed_time(t_end)
     enc_ms = [e0.elapsed_time(e1) for e0, e1 in enc_events]
-    if world > 1:
+    if sharded:
         tt = torch.tensor([ms], dtype=torch.float64, device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
@@ -316,7 +318,7 @@ def main():
         "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": C,
                    "min_match": 4, "max_match": 259, "chunks_per_gpu": ws.N,
                    "parallelism": f"dp{world} (contiguous chunk shards, NCCL all-gather of sizes)"
-                   if world > 1 else "1 GPU",
+                   if sharded else "1 GPU",
                    "l2": "inputs (256 MiB/GPU) larger than L2 (126 MB); no flush",
                    "compression_ratio": round(cr, 4), "raw_chunk_fraction": round(float(raw.mean()), 4)},
         "roofline": {"bound": "hbm", "kernel": "lzr_encode_kernel",
@@ -349,7 +351,7 @@ def main():
             e2e_t.append(time.perf_counter() - t0)
         e2e_s = statistics.median(e2e_t)
         e2e_v = n_rank / e2e_s / 1e9
-        if world > 1:
+        if sharded:
             tt = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             e2e_v = n_glob / float(tt.item()) / 1e9
@@ -365,7 +367,7 @@ def main():
                                             a.cpu_sample_bytes)
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if sharded:
         dist.destroy_process_group()
 
 
