@@ -41,9 +41,10 @@ namespace {
 
 constexpr uint16_t kFirst = 0x8000;  // first entry of its bucket
 constexpr uint16_t kPos = 0x7FFF;
-constexpr uint32_t kMaxRuns = 32;  // runs of one byte value of length >= k, per chunk
+constexpr uint32_t kMaxRuns = kMaxRunsL;  // runs of one byte value of length >= k, per chunk
 
-// ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K], T[K], M[K]
+// ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K] during
+// the walk, reused as T[K], M[K] (token / match totals) after the chain phase
 constexpr int kCtrlChunk = 0, kCtrlU = 1, kCtrlRuns = 2, kCtrlProg = 4;
 
 // Bucket of a key.  With >= 1024 buckets, keys that are one repeated byte get
@@ -217,20 +218,11 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   const bool all_in_window = p <= a.W;
   if (prun && all_in_window && nruns <= kMaxRuns)
     return best_match_runs(S, p, cap, kp, nruns, a, lane);
-  // run shortcut for the generic path (window smaller than the prefix / many runs)
-  const uint32_t rp = prun ? run_len(S.cb, p, cap) : 0u;
+  // (generic path: window smaller than the prefix, many runs, or a plain key)
+  uint32_t best = 0, blen = 0, rp = 0;
   uint32_t pw[4];
-  {
-    const uint32_t* w = reinterpret_cast<const uint32_t*>(data);
-    const uint32_t sa = (p & 3u) << 3, ia = p >> 2;
-    const uint32_t a0 = w[ia], a1 = w[ia + 1], a2 = w[ia + 2], a3 = w[ia + 3], a4 = w[ia + 4];
-    pw[0] = __funnelshift_r(a0, a1, sa);
-    pw[1] = __funnelshift_r(a1, a2, sa);
-    pw[2] = __funnelshift_r(a2, a3, sa);
-    pw[3] = __funnelshift_r(a3, a4, sa);
-  }
-  uint32_t best = 0, blen = 0;
-  int sb = (int)S.slot[p] - 1;  // the walk only asks at positions with a candidate
+  const int sb0 = (int)S.slot[p] - 1;  // the walk only asks at positions with a candidate
+  int sb = sb0;
   for (;; sb -= 32) {
     const int s = sb - (int)lane;
     uint32_t e = kFirst, q = 0;
@@ -246,11 +238,11 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
     uint32_t lim = 32;
     if (m_first) lim = (uint32_t)__ffs(m_first);
     if (m_stop) lim = min(lim, (uint32_t)(__ffs(m_stop) - 1));
-    if (lim <= 8 && blen == 0 && !rp) {
+    if (lim <= 8 && blen == 0 && !prun) {
       // few candidates (the whole list): G lanes per candidate, 4 bytes per
       // lane per step, first mismatch by ballot -- no per-lane compare loop
-      const uint32_t G = lim <= 4 ? 8u : 4u;
-      const uint32_t ci = lane / G, j = lane % G;
+      const uint32_t gs = lim <= 4 ? 3u : 2u, G = 1u << gs;
+      const uint32_t ci = lane >> gs, j = lane & (G - 1u);
       const uint32_t qc = __shfl_sync(kFull, q, ci & 31u);
       const bool act = ci < lim;
       const uint32_t gmask = ((1u << G) - 1u) << (ci * G);
@@ -274,6 +266,16 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
       uint32_t pk = 0;
       if (act && j == 0 && l >= a.m) pk = (l << 16) | (0xFFFFu - (p - qc - 1));
       return __reduce_max_sync(kFull, pk);
+    }
+    if (sb == sb0) {  // first batch of the per-lane path
+      rp = prun ? run_len(S.cb, p, cap) : 0u;
+      const uint32_t* w = reinterpret_cast<const uint32_t*>(data);
+      const uint32_t sa = (p & 3u) << 3, ia = p >> 2;
+      const uint32_t a0 = w[ia], a1 = w[ia + 1], a2 = w[ia + 2], a3 = w[ia + 3], a4 = w[ia + 4];
+      pw[0] = __funnelshift_r(a0, a1, sa);
+      pw[1] = __funnelshift_r(a1, a2, sa);
+      pw[2] = __funnelshift_r(a2, a3, sa);
+      pw[3] = __funnelshift_r(a3, a4, sa);
     }
     uint32_t pk = 0;
     if (lane < lim && (blen == 0 || data[q + blen] == data[p + blen])) {
@@ -309,12 +311,12 @@ template <int K>
 __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
                                              uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
                                              const EncArgs& a, uint32_t lane) {
-  const uint32_t nw = a.L.bm_words;
-  uint32_t* tbk = S.tb + k * nw;
-  const uint32_t* tbn = S.tb + (k + 1) * nw;  // successor's bitmap (k < K-1 only)
+  const uint32_t tw = a.L.tb_words;
+  uint32_t* tbk = S.tb + k * tw;
+  const uint32_t* tbn = S.tb + (k + 1) * tw;  // successor's bitmap (k < K-1 only)
   uint32_t* prog = S.ctrl + kCtrlProg;
   uint32_t* sync = prog + K;
-  uint32_t p = start;
+  uint32_t p = start, pub = start;
   uint32_t stop_at = n;
   while (p < n) {
     uint32_t bits = 0;
@@ -363,9 +365,12 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       }
     }
     p += tok_len ? tok_len : L;
-    if (lane == 0) {
-      __threadfence_block();
-      st_volatile(&prog[k], p);
+    if (p - pub >= 64 || p >= n) {  // publish progress (a later publish only delays meeting)
+      pub = p;
+      if (lane == 0) {
+        __threadfence_block();
+        st_volatile(&prog[k], p);
+      }
     }
   }
   if (lane == 0) sync[k] = stop_at;
@@ -386,9 +391,12 @@ __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
 }
 
 // threads per CTA at most: 10 groups of 1 or 2 warps, 9 of 3, 8 of 4
+#ifndef LZR_K4_THREADS
+#define LZR_K4_THREADS 1024
+#endif
 template <int K>
 struct MaxThreads {
-  static constexpr int value = K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : 1024));
+  static constexpr int value = K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : LZR_K4_THREADS));
 };
 
 template <int K>
@@ -408,7 +416,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
   S.cand = bms;
   S.cb = bms + nw;
   S.tb = bms + 2 * nw;
-  S.runs = bms + (2 + K) * nw;
+  S.runs = S.tb + K * a.L.tb_words;
   S.ctrl = S.runs + kMaxRuns;
   S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
   const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;
@@ -454,7 +462,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
       tma_bulk_g2s(S.data, src, n16, S.bar);
     }
     for (uint32_t i = n16 + tid; i < n; i += nthr) S.data[i] = src[i];
-    for (uint32_t i = n + tid; i < align_up(n, 16) + 32; i += nthr) S.data[i] = 0;
+    for (uint32_t i = n + tid; i < n + 20; i += nthr) S.data[i] = 0;
     uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);    // B u16 counters
     uint32_t* seen = reinterpret_cast<uint32_t*>(S.sorted);  // 2^fb-bit filter
     for (uint32_t i = tid; i < B / 2; i += nthr) hist[i] = 0;
@@ -541,7 +549,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     }
     if (K == 1 || k != 0) {
       for (uint32_t i = kk * 32 + lane; i < nw; i += KK * 32) S.cand[i] = 0;
-      for (uint32_t i = kk * 32 + lane; i < K * nw; i += KK * 32) S.tb[i] = 0;
+      for (uint32_t i = kk * 32 + lane; i < K * a.L.tb_words; i += KK * 32) S.tb[i] = 0;
       for (uint32_t w = kk; w < nw; w += KK) {  // change bitmap
         const uint32_t i = (w << 5) + lane;
         const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
@@ -651,7 +659,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         x = y;
       }
       if (in_chain && lo_k < hi_k) {
-        const uint32_t* tbk = S.tb + k * nw;
+        const uint32_t* tbk = S.tb + k * a.L.tb_words;
         for (uint32_t w = (lo_k >> 5) + lane; w <= (hi_k - 1) >> 5; w += 32) {
           uint32_t b = tbk[w];
           const uint32_t wlo = w << 5;
@@ -682,14 +690,14 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         M += __shfl_xor_sync(kFull, M, o);
       }
       if (lane == 0) {
-        S.ctrl[kCtrlProg + 2 * K + k] = T;
-        S.ctrl[kCtrlProg + 3 * K + k] = M;
+        S.ctrl[kCtrlProg + k] = T;
+        S.ctrl[kCtrlProg + K + k] = M;
       }
     }
     GSYNC(10);
     uint32_t Ttot = 0, Mtot = 0, Tb = 0, Mb = 0;
     for (uint32_t w = 0; w < K; ++w) {
-      const uint32_t t = S.ctrl[kCtrlProg + 2 * K + w], m = S.ctrl[kCtrlProg + 3 * K + w];
+      const uint32_t t = S.ctrl[kCtrlProg + w], m = S.ctrl[kCtrlProg + K + w];
       if (w < k) {
         Tb += t;
         Mb += m;
@@ -774,8 +782,10 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     // ---- copy the staged stream to the chunk's workspace slot (16-byte stores;
     //      every d1 read happened before the last group barrier)
     const uint32_t n16o = align_up(Sz, 16);
+    const uint32_t* ob32 = reinterpret_cast<const uint32_t*>(ob);  // staging is 4-byte aligned
     for (uint32_t i = tid * 16; i < n16o; i += nthr * 16)
-      *reinterpret_cast<uint4*>(out + i) = *reinterpret_cast<const uint4*>(ob + i);
+      *reinterpret_cast<uint4*>(out + i) =
+          make_uint4(ob32[i >> 2], ob32[(i >> 2) + 1], ob32[(i >> 2) + 2], ob32[(i >> 2) + 3]);
     if (tid == 0) a.sizes[c] = Sz;
   }
 }

@@ -70,8 +70,10 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
 }
 
 // ---- encode kernel shared-memory layout (one region per group of K warps) ---
+constexpr uint32_t kMaxRunsL = 24;  // run list entries per chunk (encode.cu kMaxRuns)
+
 struct EncLayout {
-  uint32_t K, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, fbits;
+  uint32_t K, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, tb_words, fbits;
 };
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
@@ -87,18 +89,21 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K) {
   L.fbits = 5;  // raw pre-filter: 2^fbits bits inside the 2C-byte index region, <= 2^15
   while ((2u << L.fbits) <= 16 * C && L.fbits < 15) ++L.fbits;
   uint32_t B = 1u << L.hbits;
-  uint32_t o = align_up(C, 16) + 32;  // chunk bytes + zero pad for 16-byte compares
+  // chunk bytes + 20 zero bytes: 16-byte compares read up to 19 bytes past n
+  uint32_t o = align_up(C + 20, 4);
   L.off_sorted = o;
-  o = align_up(o + 2 * C, 16);  // u16 positions grouped by hash bucket, ascending
+  o += 2 * C;  // u16 positions grouped by hash bucket, ascending
   L.off_slot = o;
-  o = align_up(o + 2 * (C > B ? C : B), 16);  // u16 histogram -> cursors -> slot of each position
+  o += 2 * (C > B ? C : B);  // u16 histogram -> cursors -> slot of each position
   L.off_bm = o;
-  L.bm_words = (C + 31) / 32 + 1;  // +1: two-word funnel reads at the last position
-  // bitmaps: candidate, byte-change, K token-start; run list (32); ctrl (4 + 4K)
-  o = align_up(o + 4 * ((2 + K) * L.bm_words + 32 + 4 + 4 * K), 16);
+  L.bm_words = (C + 31) / 32 + 1;  // candidate / byte-change: +1 for two-word funnel reads
+  L.tb_words = (C + 31) / 32;      // per-segment token-start bitmaps
+  // candidate, byte-change, K token-start bitmaps; run list; ctrl (4 + 2K words)
+  o += 4 * (2 * L.bm_words + K * L.tb_words + kMaxRunsL + 4 + 2 * K);
+  o = align_up(o, 8);
   L.off_mbar = o;
-  o += 16;
-  L.per_group = align_up(o, 16);
+  o += 8;
+  L.per_group = align_up(o, 16);  // next group's chunk buffer: 16-byte aligned (TMA)
   return L;
 }
 
