@@ -84,9 +84,6 @@ __device__ unsigned long long g_phase[16][4][2];
 __device__ __forceinline__ uint32_t ld_volatile(const uint32_t* p) {
   return *reinterpret_cast<const volatile uint32_t*>(p);
 }
-__device__ __forceinline__ void st_volatile(uint32_t* p, uint32_t v) {
-  *reinterpret_cast<volatile uint32_t*>(p) = v;
-}
 
 // Common-prefix length of data[a..] and data[b..], capped at maxlen; 16 bytes
 // per step (5 aligned words per side + funnel shifts).  Overlap (a > b) is
@@ -339,7 +336,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     }
     // does this stretch meet the successor's parse?
     if (K > 1 && k + 1 < K && p + L > nb) {
-      const uint32_t pr = ld_volatile(&prog[k + 1]);
+      const uint32_t pr = atomicAdd(&prog[k + 1], 0u);  // atomic read of the successor's progress
       __threadfence_block();
       const uint32_t lo = max(p, nb), hi = min(p + L, pr);
       if (lo < hi) {
@@ -358,7 +355,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
           stop_at = x;
           if (lane == 0) {
             __threadfence_block();
-            st_volatile(&prog[k], x + 1);
+            atomicExch(&prog[k], x + 1);
           }
           break;
         }
@@ -369,7 +366,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       pub = p;
       if (lane == 0) {
         __threadfence_block();
-        st_volatile(&prog[k], p);
+        atomicExch(&prog[k], p);
       }
     }
   }
