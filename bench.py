@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--ref-sample-bytes", type=int, default=8 << 20)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-decode", action="store_true")
     return ap.parse_args()
 
 
@@ -333,6 +334,25 @@ def main():
         "clocks": clk.summary(),
         "gpu_launches": launches[0],
     }
+
+    # ---- decompression of the same batch, output GB/s
+    if not a.no_decode:
+        dout = torch.empty(n_rank, dtype=torch.uint8, device=dev)
+        derr = torch.zeros(1, dtype=torch.int32, device=dev)
+        for _ in range(a.warmup):
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
+        d0, d1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        d0.record(stream)
+        for _ in range(a.steps):
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
+        d1e.record(stream)
+        torch.cuda.synchronize()
+        dms = d0.elapsed_time(d1e) / a.steps
+        ok = int(derr.item()) == 0 and bool(torch.equal(dout, x))
+        line["decode"] = {"value": round(n_rank / (dms / 1e3) / 1e9, 3), "unit": "GB/s (output)",
+                          "ms_per_step": round(dms, 4), "round_trip": "ok" if ok else "MISMATCH"}
+        del dout
 
     # ---- end to end through the C ABI with host buffers (pinned), rank 0 view
     if not a.no_e2e:
