@@ -289,9 +289,14 @@ HostSet carve(uint8_t* base, size_t batch, const lzr_params* p) {
 }
 }  // namespace
 
+// Three buffer sets on three streams: while batch b computes, batch b-1's
+// compressed bytes go back (D2H) and batch b+1's input comes in (H2D); a set is
+// reused only after its D2H was issued on its own stream (stream order).
+constexpr int kHostSets = 3;
+
 size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
   if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
-  return 2 * align_up_z(set_bytes(batch_bytes, p), 256);
+  return kHostSets * align_up_z(set_bytes(batch_bytes, p), 256);
 }
 
 int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, void* h_out,
@@ -311,13 +316,16 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   if (batch_bytes % C) return LZR_ERR_INVALID_ARG;
   if (!aligned(d_scratch, 256)) return LZR_ERR_INVALID_ARG;
   const size_t per = align_up_z(set_bytes(batch_bytes, p), 256);
-  if (scratch_bytes < 2 * per) return LZR_ERR_CAPACITY;
-  HostSet set[2] = {carve((uint8_t*)d_scratch, batch_bytes, p),
-                    carve((uint8_t*)d_scratch + per, batch_bytes, p)};
-  cudaStream_t s[2];
-  if (cudaStreamCreateWithFlags(&s[0], cudaStreamNonBlocking) != cudaSuccess) return LZR_ERR_CUDA;
-  if (cudaStreamCreateWithFlags(&s[1], cudaStreamNonBlocking) != cudaSuccess) {
-    cudaStreamDestroy(s[0]);
+  if (scratch_bytes < kHostSets * per) return LZR_ERR_CAPACITY;
+  HostSet set[kHostSets];
+  cudaStream_t s[kHostSets];
+  int made = 0;
+  for (; made < kHostSets; ++made) {
+    set[made] = carve((uint8_t*)d_scratch + made * per, batch_bytes, p);
+    if (cudaStreamCreateWithFlags(&s[made], cudaStreamNonBlocking) != cudaSuccess) break;
+  }
+  if (made < kHostSets) {
+    for (int i = 0; i < made; ++i) cudaStreamDestroy(s[i]);
     return LZR_ERR_CUDA;
   }
   const size_t nb = (n_bytes + batch_bytes - 1) / batch_bytes;
@@ -326,12 +334,12 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   int rc = LZR_OK;
   int launches = 0;
   auto issue = [&](size_t b) -> int {
-    HostSet& h = set[b & 1];
+    HostSet& h = set[b % kHostSets];
+    cudaStream_t ss = s[b % kHostSets];
     const size_t lo = b * batch_bytes;
     const size_t len = n_bytes - lo < batch_bytes ? n_bytes - lo : batch_bytes;
     const size_t c0 = b * chunks_per_batch;
     const size_t N = (len + C - 1) / C;
-    cudaStream_t ss = s[b & 1];
     if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, ss) != cudaSuccess)
       return LZR_ERR_CUDA;
     int r = lzr_compress_chunks(h.in, len, p, h.out, batch_bytes, h.sizes, h.offs, h.total, h.ws,
@@ -343,9 +351,9 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
       return LZR_ERR_CUDA;
     return LZR_OK;
   };
-  auto finish = [&](size_t b) -> int {
-    HostSet& h = set[b & 1];
-    cudaStream_t ss = s[b & 1];
+  auto finish = [&](size_t b) -> int {  // batch b's sizes are on the host: send its bytes back
+    HostSet& h = set[b % kHostSets];
+    cudaStream_t ss = s[b % kHostSets];
     if (cudaStreamSynchronize(ss) != cudaSuccess) return LZR_ERR_CUDA;
     const size_t lo = b * batch_bytes;
     const size_t len = n_bytes - lo < batch_bytes ? n_bytes - lo : batch_bytes;
@@ -361,15 +369,16 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
     running += tb;
     return LZR_OK;
   };
+  // keep two batches in flight ahead of the one being finished
   for (size_t b = 0; b < nb && rc == LZR_OK; ++b) {
     rc = issue(b);
-    if (rc == LZR_OK && b >= 1) rc = finish(b - 1);
+    if (rc == LZR_OK && b >= kHostSets - 1) rc = finish(b - (kHostSets - 1));
   }
-  if (rc == LZR_OK) rc = finish(nb - 1);
-  if (cudaStreamSynchronize(s[0]) != cudaSuccess || cudaStreamSynchronize(s[1]) != cudaSuccess)
-    rc = rc ? rc : LZR_ERR_CUDA;
-  cudaStreamDestroy(s[0]);
-  cudaStreamDestroy(s[1]);
+  for (size_t b = nb > kHostSets - 1 ? nb - (kHostSets - 1) : 0; b < nb && rc == LZR_OK; ++b)
+    rc = finish(b);
+  for (int i = 0; i < kHostSets; ++i)
+    if (cudaStreamSynchronize(s[i]) != cudaSuccess && rc == LZR_OK) rc = LZR_ERR_CUDA;
+  for (int i = 0; i < kHostSets; ++i) cudaStreamDestroy(s[i]);
   if (h_total) *h_total = running;
   t_launches = launches;
   return rc;
