@@ -315,13 +315,26 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
   uint32_t* sync = prog + K;
   uint32_t p = start, pub = start;
   uint32_t stop_at = n;
+#ifdef LZR_PHASE_TIMING
+  long long t_bm = 0, n_bm = 0, n_it = 0;
+#endif
   while (p < n) {
+#ifdef LZR_PHASE_TIMING
+    ++n_it;
+#endif
     uint32_t bits = 0;
     if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
     uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
     uint32_t tok_len = 0, r = 0;
     if (L == 0) {  // candidate position: one token
+#ifdef LZR_PHASE_TIMING
+      const long long tb0 = clock64();
+#endif
       r = best_match(S, p, n, nruns, a, lane);
+#ifdef LZR_PHASE_TIMING
+      t_bm += clock64() - tb0;
+      ++n_bm;
+#endif
       const uint32_t l = r >> 16;
       tok_len = l >= a.m ? l : 1u;
       L = 1;
@@ -371,6 +384,13 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     }
   }
   if (lane == 0) sync[k] = stop_at;
+#ifdef LZR_PHASE_TIMING
+  if (lane == 0) {
+    atomicAdd(&g_phase[12][k & 3][0], (unsigned long long)t_bm);
+    atomicAdd(&g_phase[12][k & 3][1], (unsigned long long)n_bm);
+    atomicAdd(&g_phase[13][k & 3][1], (unsigned long long)n_it);
+  }
+#endif
 }
 
 __device__ __forceinline__ uint32_t walk_bound(uint32_t n, uint32_t k, uint32_t K) {

@@ -32,4 +32,7 @@ for i, nm in enumerate(NAMES):
     w = t[i, :, 0] / N
     z = t[i, :, 1] / N
     print(f"{i:2d} {nm:14s} " + "  ".join(f"w{k}:{w[k]:7.0f}/{z[k]:6.0f}" for k in range(4)))
-print("total work", t[:, :, 0].sum() / N / 4, "wait", t[:, :, 1].sum() / N / 4)
+print("total work", t[:12, :, 0].sum() / N / 4, "wait", t[:12, :, 1].sum() / N / 4)
+print("best_match: cycles/chunk/warp", [round(t[12, k, 0] / N) for k in range(4)],
+      "calls/chunk/warp", [round(t[12, k, 1] / N, 1) for k in range(4)],
+      "walk iterations/chunk/warp", [round(t[13, k, 1] / N, 1) for k in range(4)])
