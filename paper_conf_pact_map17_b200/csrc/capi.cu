@@ -44,15 +44,17 @@ cudaError_t dev_info(DevInfo* out) {
 
 bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
-// Warps cooperating on one chunk (K).  LZR_ENCODE_WARPS=1..4 overrides (tuning).
+// Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 above (fewer
+// chunks fit one SM's shared memory, so each gets more warps).
+// LZR_ENCODE_WARPS=1,2,3,4,8 overrides (tuning).
 uint32_t enc_warps_per_chunk(uint32_t C) {
   static int env = -1;
   if (env < 0) {
     const char* e = getenv("LZR_ENCODE_WARPS");
-    env = (e && *e >= '1' && *e <= '4') ? (*e - '0') : 0;
+    env = (e && ((*e >= '1' && *e <= '4') || *e == '8')) ? (*e - '0') : 0;
   }
   if (env > 0) return (uint32_t)env;
-  return C >= 1024 ? 4u : 1u;
+  return C > 4096 ? 8u : (C >= 1024 ? 4u : 1u);
 }
 
 }  // namespace

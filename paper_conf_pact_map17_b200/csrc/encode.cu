@@ -413,7 +413,8 @@ __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
 #endif
 template <int K>
 struct MaxThreads {
-  static constexpr int value = K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : LZR_K4_THREADS));
+  static constexpr int value =
+      K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : 1024)));
 };
 
 template <int K>
@@ -842,6 +843,7 @@ cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaSt
     case 2: return launch_k<2>(a, sm_count, smem_optin, s, launches);
     case 3: return launch_k<3>(a, sm_count, smem_optin, s, launches);
     case 4: return launch_k<4>(a, sm_count, smem_optin, s, launches);
+    case 8: return launch_k<8>(a, sm_count, smem_optin, s, launches);
     default: return cudaErrorInvalidConfiguration;
   }
 }

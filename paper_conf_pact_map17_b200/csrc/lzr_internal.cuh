@@ -78,7 +78,7 @@ struct EncLayout {
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
   uint32_t hb = 0;
-  while ((2u << hb) <= C && hb < 12) ++hb;  // largest power of two <= C, capped at 4096
+  while ((2u << hb) <= C && hb < 15) ++hb;  // largest power of two <= C (the table lives in 2C bytes)
   return hb;
 }
 
