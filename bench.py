@@ -45,7 +45,11 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="lzr", choices=["lzr", "reference"])
     ap.add_argument("--cls", default="mix")
-    ap.add_argument("--bytes-per-rank", type=int, default=PER_RANK_BYTES)
+    ap.add_argument("--config", type=int, default=2, choices=[1, 2, 3, 4, 5],
+                    help="BASELINE.json config: 1 = 1 MiB, 2 = 256 MiB/GPU (default), 3 = 1 GiB/GPU "
+                         "(with --chunk-size), 4 = 16 GiB sharded, 5 = 8 GiB unique of a 16 GiB "
+                         "dedup-2.0 stream, sharded")
+    ap.add_argument("--bytes-per-rank", type=int, default=None)
     ap.add_argument("--chunk-size", type=int, default=CHUNK)
     ap.add_argument("--cpu-sample-bytes", type=int, default=24 << 20)
     ap.add_argument("--ref-sample-bytes", type=int, default=8 << 20)
@@ -227,16 +231,26 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
     p = lzr.Params(chunk_size=C)
-    n_rank = (a.bytes_per_rank // C) * C
-    n_glob = n_rank * world
+    # workload (BASELINE.json configs); weak = fixed bytes per GPU, strong = fixed total
+    if a.config in (1, 4, 5):
+        scaling = "strong"
+        n_glob = {1: 1 << 20, 4: 16 << 30, 5: 8 << 30}[a.config]
+        n_glob = (n_glob // C) * C
+    else:
+        scaling = "weak"
+        per = a.bytes_per_rank or (PER_RANK_BYTES if a.config == 2 else 1 << 30)
+        n_glob = (per // C) * C * world
+    if a.bytes_per_rank and scaling == "strong":
+        n_glob = (a.bytes_per_rank // C) * C * world
     stream = torch.cuda.current_stream(dev)
 
     # ---- inputs, generated on each GPU (global chunk indices of this shard)
     if sharded:
         sc = ShardedCompressor(n_glob, p, None, dev)
-        assert sc.n_local == n_rank
+        n_rank = sc.n_local
         first = sc.lo
     else:
+        n_rank = n_glob
         first = 0
     x = torch.empty(n_rank, dtype=torch.uint8, device=dev)
     synth.fill_device(x, C, a.cls, first_chunk=first)
@@ -308,19 +322,28 @@ def main():
     enc_avg_s = statistics.mean(enc_ms) / 1e3
     hbm_peak, peak_src = peaks()
     achieved = enc_algo_bytes / enc_avg_s / 1e9
-    workload = f"cfg2: {n_rank >> 20} MiB {a.cls} per GPU, C=W={C}, m=4, M=259"
+    if a.config == 2 and not a.bytes_per_rank:
+        workload = f"cfg2: {n_rank >> 20} MiB {a.cls} per GPU, C=W={C}, m=4, M=259"
+    elif a.config == 5:
+        workload = (f"cfg5: {n_glob >> 20} MiB unique {a.cls} chunks of a {2 * n_glob >> 20} MiB "
+                    f"dedup-2.0 stream, sharded, C=W={C}, m=4, M=259")
+    else:
+        workload = (f"cfg{a.config}: {n_glob >> 20} MiB {a.cls} total ({scaling} scaling), "
+                    f"C=W={C}, m=4, M=259")
     traffic = traffic_from_profiles(workload)
 
     line = {
         "metric": METRIC, "value": round(value, 4), "unit": UNIT, "n_gpus": world,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 4),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+        "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
         "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": C,
                    "min_match": 4, "max_match": 259, "chunks_per_gpu": ws.N,
                    "parallelism": f"dp{world} (contiguous chunk shards, NCCL all-gather of sizes)"
                    if sharded else "1 GPU",
-                   "l2": "inputs (256 MiB/GPU) larger than L2 (126 MB); no flush",
+                   "l2": (f"input ({n_rank >> 20} MiB/GPU) larger than L2 (126 MB); no flush"
+                          if n_rank > (126 << 20) else
+                          f"input ({n_rank >> 20} MiB/GPU) fits L2; no flush (small config)"),
                    "compression_ratio": round(cr, 4), "raw_chunk_fraction": round(float(raw.mean()), 4)},
         "roofline": {"bound": "hbm", "kernel": "lzr_encode_kernel",
                      "achieved": round(achieved, 3), "peak": hbm_peak, "unit": "GB/s",
@@ -356,12 +379,14 @@ def main():
 
     # ---- end to end through the C ABI with host buffers (pinned), rank 0 view
     if not a.no_e2e:
-        hx = x.cpu().pin_memory()
+        n_e2e = min(n_rank, 1 << 30)  # bounded host buffers for the big configs
+        hx = x[:n_e2e].cpu().pin_memory()
         scratch = torch.empty(max(256, lzr.lib().lzr_compress_host_scratch_bytes(
             32 << 20, __import__("ctypes").byref(p.c()))), dtype=torch.uint8, device=dev)
-        h_out = torch.empty(n_rank, dtype=torch.uint8, pin_memory=True)
-        h_sizes = torch.empty(ws.N, dtype=torch.int32, pin_memory=True)
-        h_offs = torch.empty(ws.N, dtype=torch.int64, pin_memory=True)
+        n_e2e_chunks = -(-n_e2e // C)
+        h_out = torch.empty(n_e2e, dtype=torch.uint8, pin_memory=True)
+        h_sizes = torch.empty(n_e2e_chunks, dtype=torch.int32, pin_memory=True)
+        h_offs = torch.empty(n_e2e_chunks, dtype=torch.int64, pin_memory=True)
         lzr.compress_host(hx, p, 32 << 20, scratch, h_out, h_sizes, h_offs)  # warm-up
         e2e_t = []
         for _ in range(max(1, min(a.steps, 5))):
@@ -370,21 +395,27 @@ def main():
             _, _, _, tot = lzr.compress_host(hx, p, 32 << 20, scratch, h_out, h_sizes, h_offs)
             e2e_t.append(time.perf_counter() - t0)
         e2e_s = statistics.median(e2e_t)
-        e2e_v = n_rank / e2e_s / 1e9
+        e2e_v = n_e2e / e2e_s / 1e9
         if sharded:
             tt = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            e2e_v = n_glob / float(tt.item()) / 1e9
-        line["e2e"] = {"value": round(e2e_v, 4), "unit": UNIT, "h2d_bytes_per_step": n_rank,
-                       "d2h_bytes_per_step": int(tot) + 12 * ws.N,
-                       "api": "lzr_compress_host (pinned host in/out, 32 MiB batches, 3 streams)"}
+            e2e_v = n_e2e * world / float(tt.item()) / 1e9
+        line["e2e"] = {"value": round(e2e_v, 4), "unit": UNIT, "h2d_bytes_per_step": n_e2e,
+                       "d2h_bytes_per_step": int(tot) + 12 * n_e2e_chunks,
+                       "api": "lzr_compress_host (pinned host in/out, 32 MiB batches, 3 streams)"
+                              + ("" if n_e2e == n_rank else f", first {n_e2e >> 20} MiB per GPU")}
         del scratch
 
+    if a.config == 5:
+        line["logical_value"] = round(2 * value, 4)  # logical (pre-dedup) bytes per second
     if rank == 0 and not a.no_cpu:
-        g_out = ws.out[:total].cpu().numpy()
-        g_offs = ws.offsets[: ws.N].cpu().numpy().view(np.uint64)
-        line["cpu_baseline"] = cpu_baseline(x.cpu().numpy(), p, sizes, g_offs, g_out,
-                                            a.cpu_sample_bytes)
+        smp = min(n_rank, (a.cpu_sample_bytes // C) * C) if a.config != 1 else n_rank
+        ns = -(-smp // C)
+        g_offs = ws.offsets[:ns].cpu().numpy().view(np.uint64)
+        end = int(g_offs[-1]) + int(sizes[ns - 1])
+        g_out = ws.out[:end].cpu().numpy()
+        line["cpu_baseline"] = cpu_baseline(x[:smp].cpu().numpy(), p, sizes[:ns], g_offs, g_out,
+                                            smp)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if sharded:

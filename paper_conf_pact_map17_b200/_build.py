@@ -42,6 +42,13 @@ def build_timing() -> str:
     return out
 
 
+def build_watchdog() -> str:
+    """Debug variant: spin loops trap with a message after ~2^26 iterations."""
+    out = os.path.join(PKG, "liblzr_dbg.so")
+    subprocess.check_call(["nvcc", *NVCC_FLAGS, "-DLZR_WATCHDOG", "-o", out, *sources()])
+    return out
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
     if force or stale():
         cmd = ["nvcc", *NVCC_FLAGS, *(["-Xptxas", "-v"] if verbose else []),
@@ -55,6 +62,8 @@ if __name__ == "__main__":
     import sys
     if "--timing" in sys.argv:
         print(build_timing())
+    elif "--watchdog" in sys.argv:
+        print(build_watchdog())
     else:
         build(force="-f" in sys.argv, verbose="-v" in sys.argv)
         print(LIB)

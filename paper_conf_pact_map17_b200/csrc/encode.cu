@@ -318,7 +318,11 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
 #ifdef LZR_PHASE_TIMING
   long long t_bm = 0, n_bm = 0, n_it = 0;
 #endif
+#ifdef LZR_WATCHDOG
+  uint32_t spins = 0;
+#endif
   while (p < n) {
+    LZR_SPIN_GUARD(spins, "walk")
 #ifdef LZR_PHASE_TIMING
     ++n_it;
 #endif
@@ -349,13 +353,19 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     }
     // does this stretch meet the successor's parse?
     if (K > 1 && k + 1 < K && p + L > nb) {
-      const uint32_t pr = atomicAdd(&prog[k + 1], 0u);  // atomic read of the successor's progress
+      // one atomic read of the successor's progress, broadcast: per-lane reads
+      // could see different values and split the warp (-> warp-sync deadlock)
+      uint32_t pr = 0;
+      if (lane == 0) pr = atomicAdd(&prog[k + 1], 0u);
+      pr = __shfl_sync(kFull, pr, 0);
       __threadfence_block();
       const uint32_t lo = max(p, nb), hi = min(p + L, pr);
       if (lo < hi) {
         uint32_t x = hi;
         for (uint32_t w = lo >> 5; w <= (hi - 1) >> 5; ++w) {
-          uint32_t b = ld_volatile(&tbn[w]);
+          uint32_t b = 0;
+          if (lane == 0) b = ld_volatile(&tbn[w]);
+          b = __shfl_sync(kFull, b, 0);  // uniform across the warp (see above)
           const uint32_t wlo = w << 5;
           if (wlo < lo) b &= 0xFFFFFFFFu << (lo - wlo);
           if (hi - wlo < 32) b &= (1u << (hi - wlo)) - 1u;

@@ -4,6 +4,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdio.h>
 
 #include "../../include/lzr.h"
 
@@ -56,9 +57,23 @@ __device__ __forceinline__ void tma_bulk_g2s(void* smem_dst, const void* gmem_sr
       "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+#ifdef LZR_WATCHDOG
+#define LZR_SPIN_GUARD(cnt, what)                                                          \
+  if (++(cnt) == (1u << 20)) {                                                             \
+    printf("lzr watchdog: %s stuck, block %d thread %d\n", what, blockIdx.x, threadIdx.x); \
+    __trap();                                                                              \
+  }
+#else
+#define LZR_SPIN_GUARD(cnt, what)
+#endif
+
 __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity) {
   uint32_t done = 0;
+#ifdef LZR_WATCHDOG
+  uint32_t spins = 0;
+#endif
   while (!done) {
+    LZR_SPIN_GUARD(spins, "mbarrier wait")
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
         "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"

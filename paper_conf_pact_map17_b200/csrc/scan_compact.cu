@@ -74,7 +74,11 @@ __global__ void __launch_bounds__(kScanThreads) lzr_scan_kernel(const uint32_t* 
         const long idx = j - (long)lane;
         uint64_t st = 0;
         if (idx >= 0) {
+#ifdef LZR_WATCHDOG
+          uint32_t spins = 0;
+#endif
           do {
+            LZR_SPIN_GUARD(spins, "scan look-back")
             st = ld_status(&status[idx]);
           } while ((st >> 62) == 0);
         } else {

@@ -232,3 +232,26 @@ def test_empty_input(lzr):
     out, sizes, offs, total = lzr.compress(xd, lzr.Params())
     torch.cuda.synchronize()
     assert sizes.numel() == 0 and int(total.item()) == 0
+
+
+@pytest.mark.timeout(300)
+@pytest.mark.parametrize("C", [4096, 8192])
+def test_repeated_launch_stress(lzr, C):
+    """Many back-to-back launches on one workspace (a lane-divergent progress read
+    once split warps in the speculative walk and deadlocked a warp-sync; this
+    exercises the meeting logic under varying timing).  Results must be stable."""
+    p = lzr.Params(chunk_size=C)
+    n = 256 << 20
+    xd = torch.empty(n, dtype=torch.uint8, device="cuda")
+    synth.fill_device(xd, C, "mix", seed=C)
+    ws = lzr.Workspace(n, p, xd.device)
+    ref_total = None
+    for i in range(12):
+        out, sizes, offs, total = lzr.compress(xd, p, ws=ws)
+        torch.cuda.synchronize()
+        t = int(total.item())
+        ref_total = t if ref_total is None else ref_total
+        assert t == ref_total
+    y, err = lzr.decompress(out, sizes, offs, n, p)
+    torch.cuda.synchronize()
+    assert int(err.item()) == 0 and torch.equal(y, xd)
