@@ -81,6 +81,10 @@ __device__ unsigned long long g_phase[16][4][2];
 #define GSYNC(ph) group_sync(bar_id, nthr)
 #endif
 
+__device__ __forceinline__ void fence_acq_rel_cta() {
+  asm volatile("fence.acq_rel.cta;" ::: "memory");
+}
+
 __device__ __forceinline__ uint32_t ld_volatile(const uint32_t* p) {
   return *reinterpret_cast<const volatile uint32_t*>(p);
 }
@@ -356,9 +360,11 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       // one atomic read of the successor's progress, broadcast: per-lane reads
       // could see different values and split the warp (-> warp-sync deadlock)
       uint32_t pr = 0;
-      if (lane == 0) pr = atomicAdd(&prog[k + 1], 0u);
+      if (lane == 0) {
+        pr = atomicAdd(&prog[k + 1], 0u);
+        fence_acq_rel_cta();  // the successor's bits below pr are visible after this
+      }
       pr = __shfl_sync(kFull, pr, 0);
-      __threadfence_block();
       const uint32_t lo = max(p, nb), hi = min(p + L, pr);
       if (lo < hi) {
         uint32_t x = hi;
@@ -377,7 +383,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
         if (x < hi) {
           stop_at = x;
           if (lane == 0) {
-            __threadfence_block();
+            fence_acq_rel_cta();
             atomicExch(&prog[k], x + 1);
           }
           break;
@@ -388,7 +394,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     if (p - pub >= 64 || p >= n) {  // publish progress (a later publish only delays meeting)
       pub = p;
       if (lane == 0) {
-        __threadfence_block();
+        fence_acq_rel_cta();  // recorded token bits before the progress word
         atomicExch(&prog[k], p);
       }
     }
