@@ -81,6 +81,23 @@ __device__ unsigned long long g_phase[16][4][2];
 #define GSYNC(ph) group_sync(bar_id, nthr)
 #endif
 
+// predicated shared-memory OR without a returned value (no branch, no wait)
+__device__ __forceinline__ void red_or_if(bool pred, uint32_t* addr, uint32_t v) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %0, 0;\n\t@q red.shared.or.b32 [%1], %2;\n\t}" ::"r"(
+          (uint32_t)pred),
+      "r"(smem_u32(addr)), "r"(v)
+      : "memory");
+}
+// predicated 16-bit global store
+__device__ __forceinline__ void st_u16_if(bool pred, uint16_t* addr, uint32_t v) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %0, 0;\n\t@q st.global.u16 [%1], %2;\n\t}" ::"r"(
+          (uint32_t)pred),
+      "l"(addr), "h"((uint16_t)v)
+      : "memory");
+}
+
 __device__ __forceinline__ void fence_acq_rel_cta() {
   asm volatile("fence.acq_rel.cta;" ::: "memory");
 }
@@ -347,13 +364,13 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       tok_len = l >= a.m ? l : 1u;
       L = 1;
     }
-    // record token starts [p, p+L)
-    if (lane == 0) {
+    // record token starts [p, p+L) and (d-1) (lane 0 / lane 1, predicated)
+    {
       const uint32_t w = p >> 5, sh = p & 31u;
       const uint32_t mask = L >= 32 ? 0xFFFFFFFFu : ((1u << L) - 1u);
-      atomicOr(&tbk[w], mask << sh);
-      if (sh + L > 32) atomicOr(&tbk[w + 1], mask >> (32 - sh));
-      if (tok_len > 1) d1[p] = (uint16_t)(0xFFFFu - (r & 0xFFFFu));  // d - 1
+      red_or_if(lane == 0, &tbk[w], mask << sh);
+      red_or_if(lane == 0 && sh + L > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
+      st_u16_if(lane == 0 && tok_len > 1, d1 + p, 0xFFFFu - (r & 0xFFFFu));  // d - 1
     }
     // does this stretch meet the successor's parse?
     if (K > 1 && k + 1 < K && p + L > nb) {
