@@ -187,7 +187,8 @@ int lzr_compress_compact(const void* d_in, size_t n_bytes, const lzr_params* p, 
   if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
   const size_t N = (n_bytes + p->chunk_size - 1) / p->chunk_size;
   uint8_t* ws = (uint8_t*)d_workspace;
-  if (launch_scan(d_sizes, N, 0, d_offsets, d_total, ws + w.scan_off, s, &t_launches) != cudaSuccess)
+  if (launch_scan(d_sizes, N, 0, nullptr, d_offsets, d_total, ws + w.scan_off, s, &t_launches) !=
+      cudaSuccess)
     return LZR_ERR_CUDA;
   if (launch_compact((const uint8_t*)d_in, n_bytes, p->chunk_size, ws + w.slots_off,
                      (size_t)p->chunk_size, d_sizes,
@@ -232,7 +233,8 @@ int lzr_scan_sizes(const uint32_t* d_sizes, size_t n, uint64_t base, uint64_t* d
       (d_total && !aligned(d_total, 8)))
     return LZR_ERR_INVALID_ARG;
   if (workspace_bytes < scan_ws_bytes(n)) return LZR_ERR_CAPACITY;
-  if (launch_scan(d_sizes, n, base, d_offsets, d_total, d_workspace, s, &t_launches) != cudaSuccess)
+  if (launch_scan(d_sizes, n, base, nullptr, d_offsets, d_total, d_workspace, s, &t_launches) !=
+      cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;
 }

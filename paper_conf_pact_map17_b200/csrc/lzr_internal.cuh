@@ -145,8 +145,9 @@ WsLayout ws_layout(size_t n_bytes, const lzr_params* p);
 
 // launches (defined in the .cu files); return cudaError_t of the launch
 cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches);
-cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, uint64_t* offsets,
-                        uint64_t* total, void* ws, cudaStream_t s, int* launches);
+cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, const uint64_t* base_ptr,
+                        uint64_t* offsets, uint64_t* total, void* ws, cudaStream_t s,
+                        int* launches);
 cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const uint8_t* slots,
                            size_t slot_stride,
                            const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,

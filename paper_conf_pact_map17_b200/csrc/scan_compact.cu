@@ -29,8 +29,10 @@ __device__ __forceinline__ void st_status(uint64_t* p, uint64_t v) {
 // ws: [0] u32 tile counter; [256..) u64 status per tile.  Zeroed before launch.
 __global__ void __launch_bounds__(kScanThreads) lzr_scan_kernel(const uint32_t* __restrict__ sizes,
                                                                size_t n, uint64_t base,
+                                                               const uint64_t* base_ptr,
                                                                uint64_t* __restrict__ offsets,
                                                                uint64_t* total, uint8_t* ws) {
+  if (base_ptr) base += *base_ptr;  // device-side running base (chained batches)
   __shared__ uint32_t s_tile;
   __shared__ uint64_t s_warp[kScanThreads / 32];
   __shared__ uint64_t s_prefix;
@@ -109,27 +111,35 @@ __global__ void __launch_bounds__(kScanThreads) lzr_scan_kernel(const uint32_t* 
 }
 
 // Copy S bytes src -> dst (dst arbitrary alignment, src 16-byte aligned chunk
-// base) with one warp: byte head up to a 4-byte boundary of dst, funnel-shifted
-// 32-bit body, byte tail.  Reads stay inside [src, src + S).
+// base) with one warp: bytes up to a 16-byte boundary of dst, then 16-byte
+// stores assembled from funnel-shifted source words (full-line writes also when
+// dst is pinned host memory written over PCIe), then the byte tail.  Reads stay
+// inside [src, src + S).
 __device__ __forceinline__ void warp_copy(uint8_t* dst, const uint8_t* src, uint32_t S,
                                           uint32_t lane) {
-  uint32_t head = (4u - (uint32_t)((uintptr_t)dst & 3u)) & 3u;
+  uint32_t head = (16u - (uint32_t)((uintptr_t)dst & 15u)) & 15u;
   if (head > S) head = S;
   if (lane < head) dst[lane] = src[lane];
-  const uint32_t a = head & 3u;  // src misalignment of the body (src base is aligned)
+  const uint32_t a = head & 3u;  // byte misalignment of the body's source
   const uint32_t sw = head >> 2;
   const uint32_t full = S >> 2;  // whole source words
-  long nb = ((long)S - (long)head) >> 2;
-  const long lim = (long)full - (long)sw - (a ? 1 : 0);
-  if (nb > lim) nb = lim;
-  if (nb < 0) nb = 0;
+  // 16-byte output vectors whose 4 (or 5 when misaligned) source words are whole
+  long nv = ((long)S - (long)head) >> 4;
+  const long lim = ((long)full - (long)sw - (a ? 1 : 0)) >> 2;
+  if (nv > lim) nv = lim;
+  if (nv < 0) nv = 0;
   const uint32_t* s32 = reinterpret_cast<const uint32_t*>(src);
-  uint32_t* d32 = reinterpret_cast<uint32_t*>(dst + head);
-  for (long k = lane; k < nb; k += 32) {
-    const uint32_t w0 = s32[sw + k];
-    d32[k] = a ? __funnelshift_r(w0, s32[sw + k + 1], a << 3) : w0;
+  uint4* d128 = reinterpret_cast<uint4*>(dst + head);
+  const uint32_t sh = a << 3;
+  for (long k = lane; k < nv; k += 32) {
+    const uint32_t w = sw + 4 * (uint32_t)k;
+    const uint32_t w0 = s32[w], w1 = s32[w + 1], w2 = s32[w + 2], w3 = s32[w + 3];
+    const uint32_t w4 = a ? s32[w + 4] : 0u;
+    d128[k] = a ? make_uint4(__funnelshift_r(w0, w1, sh), __funnelshift_r(w1, w2, sh),
+                             __funnelshift_r(w2, w3, sh), __funnelshift_r(w3, w4, sh))
+                : make_uint4(w0, w1, w2, w3);
   }
-  for (uint32_t i = head + (uint32_t)nb * 4u + lane; i < S; i += 32) dst[i] = src[i];
+  for (uint32_t i = head + (uint32_t)nv * 16u + lane; i < S; i += 32) dst[i] = src[i];
 }
 
 __global__ void __launch_bounds__(256) lzr_compact_kernel(const uint8_t* __restrict__ in,
@@ -158,14 +168,15 @@ size_t scan_ws_bytes(size_t n) {
   return align_up_z(256 + ntiles * 8, 256);
 }
 
-cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, uint64_t* offsets,
-                        uint64_t* total, void* ws, cudaStream_t s, int* launches) {
+cudaError_t launch_scan(const uint32_t* sizes, size_t n, uint64_t base, const uint64_t* base_ptr,
+                        uint64_t* offsets, uint64_t* total, void* ws, cudaStream_t s,
+                        int* launches) {
   cudaError_t err = cudaMemsetAsync(ws, 0, scan_ws_bytes(n), s);
   if (err != cudaSuccess) return err;
   const size_t ntiles = (n + kScanTile - 1) / kScanTile;
   if (ntiles == 0) return cudaSuccess;
-  lzr_scan_kernel<<<(unsigned)ntiles, kScanThreads, 0, s>>>(sizes, n, base, offsets, total,
-                                                            (uint8_t*)ws);
+  lzr_scan_kernel<<<(unsigned)ntiles, kScanThreads, 0, s>>>(sizes, n, base, base_ptr, offsets,
+                                                            total, (uint8_t*)ws);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
