@@ -251,7 +251,7 @@ int lzr_decompress_chunks(const void* d_comp, const uint32_t* d_sizes, const uin
   if (n_bytes && (!aligned(d_sizes, 4) || !aligned(d_offsets, 8))) return LZR_ERR_INVALID_ARG;
   DevInfo di;
   if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
-  if ((int)(align_up(p->chunk_size, 16) + align_up(p->chunk_size + 8, 16)) > di.smem_optin)
+  if ((int)align_up(p->chunk_size, 16) > di.smem_optin)
     return LZR_ERR_UNSUPPORTED;
   if (launch_decode((const uint8_t*)d_comp, d_sizes, d_offsets, n_bytes, p->chunk_size,
                     p->min_match, (uint8_t*)d_out, d_error, di.sm_count, di.smem_optin, s,

@@ -1,14 +1,18 @@
-// decode.cu -- inverse of the encoder (R1, R5, R9): one warp per chunk.
+// decode.cu -- inverse of the encoder (R1, R5, R9): one warp per chunk, 32
+// tokens (four flag-byte groups) per step.
 //
-// The chunk's compressed stream is first staged into shared memory with
-// aligned 4-byte loads (one coalesced pass), so every later header/token read
-// is a shared-memory access.  Per flag-byte group, lanes 0..7 read the eight
-// token headers in parallel (token j starts at ip + j + 2*popc(flags below j)),
-// an 8-lane prefix sum of token lengths gives their output positions, literals
-// are written in parallel, then matches are expanded in order, each by the
-// whole warp: out[o + k] = out[o - d + (k mod d)] only reads bytes before o,
-// which are final, so overlapping matches (d < l) need no byte-serial loop.
-// The chunk is rebuilt in shared memory and written out with 16-byte stores;
+// The four flag bytes of a step are a short dependent chain (group g + 1
+// starts 9 + 2 popc(f_g) bytes after group g); then lane t owns token t: its
+// stream offset is ip_g + 1 + j + 2 popc(f_g below j), its output position a
+// 32-lane prefix sum of token lengths.  Token headers are read straight from
+// global memory (L1-cached byte loads, never outside [src, src + S)).  The chunk
+// is rebuilt in shared memory: literals of the step are stored in parallel,
+// then the step's matches are resolved in rounds -- a match whose source bytes
+// lie below the first unresolved match's output (or that is the first one) is
+// final-sourced, so all such matches copy at once: short ones one lane each,
+// byte-serially (which also gives overlapping matches, d < l, their R5
+// meaning), long ones by the whole warp (out[o + k] = out[o - d + (k mod d)]
+// only reads bytes before o).  The chunk is written out with 16-byte stores;
 // raw chunks are copied with 16-byte stores from funnel-shifted 4-byte loads.
 // Malformed streams set *err = min(1 + chunk index) (err pre-set to 0x7F7F7F7F,
 // fixed up to 0 afterwards when no chunk was corrupt).
@@ -18,8 +22,9 @@ namespace lzr {
 
 namespace {
 
-constexpr int kDecWarpsMax = 8;
+constexpr int kDecWarpsMax = 16;
 constexpr int32_t kNoError = 0x7F7F7F7F;
+constexpr uint32_t kLaneCopyMax = 16;  // matches up to this length: one lane, byte-serial
 
 __device__ int32_t g_scratch_err;
 
@@ -37,26 +42,22 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
   return v;
 }
 
-// Stage src[0..S) (arbitrary alignment) into smem: buf + (src & 3) holds src[0].
-__device__ __forceinline__ const uint8_t* stage_stream(uint8_t* buf, const uint8_t* src, uint32_t S,
-                                                       uint32_t lane) {
-  const uint32_t mis = (uint32_t)((uintptr_t)src & 3u);
-  uint32_t* b32 = reinterpret_cast<uint32_t*>(buf);
-  const uint32_t words = (mis + S + 3) >> 2;
-  for (uint32_t i = lane; i < words; i += 32) b32[i] = load_word(src, mis, S, i);
-  return buf + mis;
+// stream byte x, 0 past the end (the caller flags the error)
+__device__ __forceinline__ uint32_t sbyte(const uint8_t* src, uint32_t S, uint32_t x) {
+  return x < S ? (uint32_t)__ldg(src + x) : 0u;
 }
 
-__global__ void __launch_bounds__(32 * kDecWarpsMax, 1) lzr_decode_kernel(
+__global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
     const uint8_t* __restrict__ comp, const uint32_t* __restrict__ sizes,
     const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C, uint32_t m,
     uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride) {
   extern __shared__ __align__(16) uint8_t dsm[];
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   uint8_t* obuf = dsm + (size_t)warp * buf_stride;  // rebuilt chunk (C bytes)
-  uint8_t* sbuf = obuf + align_up(C, 16);           // staged stream (C + 4 bytes)
   const size_t gw = (size_t)blockIdx.x * (blockDim.x >> 5) + warp;
   const size_t nw = (size_t)gridDim.x * (blockDim.x >> 5);
+  const uint32_t g = lane >> 3, j = lane & 7u;
+  const uint32_t below = (1u << j) - 1u;
   for (size_t c = gw; c < N; c += nw) {
     const size_t lo = c * C;
     const uint32_t n = (uint32_t)min((size_t)C, n_bytes - lo);
@@ -80,68 +81,91 @@ __global__ void __launch_bounds__(32 * kDecWarpsMax, 1) lzr_decode_kernel(
       continue;
     }
     bool bad = S > n;
-    const uint8_t* s = bad ? sbuf : stage_stream(sbuf, src, S, lane);
-    __syncwarp();
     uint32_t ip = 0, op = 0;
     while (!bad && op < n) {
-      if (ip >= S) {
-        bad = true;
-        break;
+      // the four groups of this step: flag byte and stream offset
+      uint32_t f = 0, ipg = 0;
+      {
+        uint32_t x = ip;
+#pragma unroll
+        for (uint32_t t = 0; t < 4; ++t) {
+          const uint32_t ft = sbyte(src, S, x);
+          if (t == g) {
+            f = ft;
+            ipg = x;
+          }
+          x += 9u + 2u * __popc(ft);
+        }
       }
-      const uint32_t f = s[ip];
-      ip += 1;
-      const uint32_t j = lane & 7u;
       const uint32_t ism = (f >> j) & 1u;
-      const uint32_t toff = ip + j + 2u * __popc(f & ((1u << j) - 1u));
+      const uint32_t toff = ipg + 1u + j + 2u * __popc(f & below);
       const uint32_t tsz = 1u + 2u * ism;
-      const uint32_t b0 = toff < S ? s[toff] : 0u;
+      const uint32_t b0 = sbyte(src, S, toff);
       uint32_t b1 = 0, b2 = 0;
       if (ism) {
-        b1 = toff + 1 < S ? s[toff + 1] : 0u;
-        b2 = toff + 2 < S ? s[toff + 2] : 0u;
+        b1 = sbyte(src, S, toff + 1);
+        b2 = sbyte(src, S, toff + 2);
       }
       const uint32_t tlen = ism ? b2 + m : 1u;
       const uint32_t d = (b0 | (b1 << 8)) + 1u;
       uint32_t incl = tlen;
 #pragma unroll
-      for (int o = 1; o < 8; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(kFull, incl, o, 8);
-        if ((int)j >= o) incl += t;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(kFull, incl, o);
+        if ((int)lane >= o) incl += t;
       }
-      const uint32_t ob = op + incl - tlen;  // output position of token j
-      const bool reached = ob < n;
+      const uint32_t ob = op + incl - tlen;  // output position of token `lane`
+      // a group is live when the groups before it did not finish the chunk
+      const uint32_t gstart = __shfl_sync(kFull, ob, lane & ~7u);
+      const bool live = gstart < n;
+      const bool reached = live && ob < n;
       bool e = false;
+      if (live && ipg >= S) e = true;  // flag byte past the stream
       if (reached) {
         if (toff + tsz > S) e = true;
         if (ism && (d > ob || ob + tlen > n)) e = true;
-      } else if (ism) {
+      } else if (live && ism) {
         e = true;  // padding flag bits must be zero
       }
-      if (__ballot_sync(kFull, lane < 8 && e)) {
+      if (__any_sync(kFull, e)) {
         bad = true;
         break;
       }
-      const uint32_t rmask = __ballot_sync(kFull, lane < 8 && reached);
-      const uint32_t nt = __popc(rmask);
-      const uint32_t fr = f & rmask;
-      if (lane < 8 && reached && !ism) obuf[ob] = (uint8_t)b0;
+      const uint32_t rmask = __ballot_sync(kFull, reached);  // a prefix of the lanes
+      const uint32_t last = 31u - __clz(rmask);
+      if (reached && !ism) obuf[ob] = (uint8_t)b0;
       __syncwarp();
-      uint32_t mm = fr;
-      while (mm) {
-        const int jj = __ffs(mm) - 1;
-        mm &= mm - 1;
-        const uint32_t o = __shfl_sync(kFull, ob, jj);
-        const uint32_t dd = __shfl_sync(kFull, d, jj);
-        const uint32_t ll = __shfl_sync(kFull, tlen, jj);
-        if (dd >= ll) {
-          for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + k];
-        } else {
-          for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + (k % dd)];
+      uint32_t pend = __ballot_sync(kFull, reached && ism);
+      // bytes a match needs before its own output (the rest overlaps itself)
+      const uint32_t need_end = ob - d + min(tlen, d);
+      while (pend) {
+        const uint32_t f0 = (uint32_t)(__ffs(pend) - 1);
+        const uint32_t first_ob = __shfl_sync(kFull, ob, f0);
+        const bool mine = (pend >> lane) & 1u;
+        const uint32_t ready = __ballot_sync(kFull, mine && (lane == f0 || need_end <= first_ob));
+        const bool go = (ready >> lane) & 1u;
+        if (go && tlen <= kLaneCopyMax) {
+          for (uint32_t k = 0; k < tlen; ++k) obuf[ob + k] = obuf[ob - d + k];
+        }
+        uint32_t lng = ready & __ballot_sync(kFull, tlen > kLaneCopyMax);
+        while (lng) {
+          const int jj = __ffs(lng) - 1;
+          lng &= lng - 1;
+          const uint32_t o = __shfl_sync(kFull, ob, jj);
+          const uint32_t dd = __shfl_sync(kFull, d, jj);
+          const uint32_t ll = __shfl_sync(kFull, tlen, jj);
+          if (dd >= ll) {
+            for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + k];
+          } else {
+            for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + (k % dd)];
+          }
+          __syncwarp();
         }
         __syncwarp();
+        pend &= ~ready;
       }
-      op += __shfl_sync(kFull, incl, nt - 1);
-      ip += nt + 2u * __popc(fr);
+      op = __shfl_sync(kFull, ob + tlen, last);
+      ip = __shfl_sync(kFull, toff + tsz, last);
     }
     if (!bad && ip != S) bad = true;
     if (bad) {
@@ -172,7 +196,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
     if (err) return cudaMemsetAsync(err, 0, sizeof(int32_t), s);
     return cudaSuccess;
   }
-  const uint32_t stride = align_up(C, 16) + align_up(C + 8, 16);  // rebuilt chunk + staged stream
+  const uint32_t stride = align_up(C, 16);  // rebuilt chunk
   int warps = smem_optin / (int)stride;
   if (warps > kDecWarpsMax) warps = kDecWarpsMax;
   if (warps < 1) return cudaErrorInvalidConfiguration;

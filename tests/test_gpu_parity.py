@@ -255,3 +255,64 @@ def test_repeated_launch_stress(lzr, C):
     y, err = lzr.decompress(out, sizes, offs, n, p)
     torch.cuda.synchronize()
     assert int(err.item()) == 0 and torch.equal(y, xd)
+
+
+def _mutate(rng, s: bytes, n: int) -> bytes:
+    """One random corruption (or a random valid-looking edit) of a chunk stream."""
+    b = bytearray(s)
+    kind = int(rng.integers(0, 7))
+    if kind == 0 and b:  # flip a bit
+        i = int(rng.integers(0, len(b)))
+        b[i] ^= 1 << int(rng.integers(0, 8))
+    elif kind == 1 and b:  # a flag byte (the first) to a random value
+        b[0] = int(rng.integers(0, 256))
+    elif kind == 2 and len(b) > 1:  # truncate
+        b = b[: int(rng.integers(0, len(b)))]
+    elif kind == 3:  # trailing garbage
+        b += bytes(rng.integers(0, 256, int(rng.integers(1, 4)), dtype=np.uint8))
+    elif kind == 4:  # random stream of random length (< n: not raw)
+        b = bytearray(rng.integers(0, 256, int(rng.integers(1, n)), dtype=np.uint8))
+    elif kind == 5 and len(b) > 3:  # a length / distance byte to an extreme
+        i = int(rng.integers(1, len(b)))
+        b[i] = 0xFF if rng.integers(0, 2) else 0x00
+    else:  # all flags set in the first group
+        if b:
+            b[0] = 0xFF
+    if len(b) >= n:  # keep it a "compressed" chunk (size == n means raw)
+        b = b[: n - 1]
+    return bytes(b)
+
+
+@pytest.mark.parametrize("C,m,cls", [(4096, 4, "text"), (4096, 4, "zeroruns"), (1024, 3, "cr2"),
+                                     (256, 9, "text")])
+def test_gpu_decoder_fuzz_vs_oracle(lzr, ref, C, m, cls):
+    """Random corruptions of 1-3 chunks per trial: the GPU decoder's verdict
+    (first bad chunk) equals the oracle decoder's; when every chunk is still
+    valid, the outputs are equal byte for byte."""
+    nch = 24
+    x = synth.fill_host(nch * C - 77, C, cls, seed=C + m)
+    p = lzr.Params(chunk_size=C, min_match=m)
+    rp = _ref_params(ref, p)
+    _, _, _, _, _, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, p)
+    streams = [g_out[g_offs[i]: g_offs[i] + g_sizes[i]].tobytes() for i in range(g_sizes.size)]
+    ns = [min(C, x.size - i * C) for i in range(g_sizes.size)]
+    comp_ok = [i for i in range(len(streams)) if g_sizes[i] < ns[i]]
+    assert comp_ok, "need compressed chunks"
+    rng = np.random.default_rng(C * 31 + m)
+    n_valid = 0
+    for trial in range(60):
+        ss = list(streams)
+        for ci in rng.choice(comp_ok, size=int(rng.integers(1, 4)), replace=False):
+            ss[int(ci)] = _mutate(rng, ss[int(ci)], ns[int(ci)])
+        sizes = np.array([len(s) for s in ss], np.uint32)
+        offs = np.concatenate([[0], np.cumsum(sizes[:-1], dtype=np.uint64)]).astype(np.uint64)
+        comp = np.frombuffer(b"".join(ss) + b"\0", np.uint8)
+        st, r_bad, r_y = ref.decompress(comp, sizes, offs, x.size, rp)
+        y, err = lzr.decompress(torch.from_numpy(comp.copy()).cuda(),
+                                torch.from_numpy(sizes.view(np.int32)).cuda(),
+                                torch.from_numpy(offs.view(np.int64)).cuda(), x.size, p)
+        torch.cuda.synchronize()
+        assert int(err.item()) == r_bad, (trial, r_bad)
+        if r_bad == 0:
+            n_valid += 1
+            assert np.array_equal(y.cpu().numpy(), r_y), trial
