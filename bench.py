@@ -182,7 +182,7 @@ def run_reference(a):
     times = []
     for step in range(a.warmup + a.steps):
         # each step a different bounded sample of the workload stream
-        first = (step * (n // C)) % max(1, (a.bytes_per_rank // C))
+        first = (step * (n // C)) % max(1, ((a.bytes_per_rank or PER_RANK_BYTES) // C))
         x = synth.fill_host(n, C, a.cls, first_chunk=first)
         t0 = time.perf_counter()
         oracle.compress(x, p, n_threads=cores)
