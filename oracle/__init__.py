@@ -19,6 +19,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "liblzr_ref.so")
+DEDUP_LIB_PATH = os.path.join(_HERE, "liblzr_dedup_ref.so")
 
 OK = 0
 ERR_INVALID_ARG = -1
@@ -67,6 +68,15 @@ def build(force: bool = False) -> str:
              "-o", LIB_PATH + ".tmp", src]
         )
         os.replace(LIB_PATH + ".tmp", LIB_PATH)
+    dsrc = os.path.join(_HERE, "dedup_ref.c")
+    if force or not os.path.exists(DEDUP_LIB_PATH) or os.path.getmtime(DEDUP_LIB_PATH) < os.path.getmtime(dsrc):
+        import subprocess
+
+        subprocess.check_call(
+            ["gcc", "-O2", "-std=c11", "-Wall", "-Wextra", "-fPIC", "-shared", "-pthread",
+             "-o", DEDUP_LIB_PATH + ".tmp", dsrc]
+        )
+        os.replace(DEDUP_LIB_PATH + ".tmp", DEDUP_LIB_PATH)
     return LIB_PATH
 
 
@@ -194,3 +204,71 @@ def decompress(comp, sizes, offsets, n: int, p: Params) -> tuple[int, int, np.nd
     st = lib().lzr_ref_decompress(_ptr(c), _ptr(s), _ptr(o), n, ctypes.byref(p.c()), _ptr(out),
                                   ctypes.byref(bad))
     return st, bad.value, out[:n]
+
+
+# ---- dedup (oracle/dedup_ref.c) -------------
+_dlib = None
+
+
+def dlib():
+    global _dlib
+    if _dlib is None:
+        build()
+        L = ctypes.CDLL(DEDUP_LIB_PATH)
+        L.dedup_ref_sha1.argtypes = [ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p]
+        L.dedup_ref_fingerprints.argtypes = [ctypes.c_void_p, ctypes.c_size_t, ctypes.c_size_t,
+                                             ctypes.c_void_p, ctypes.c_int]
+        _dlib = L
+    return _dlib
+
+
+def sha1(x) -> bytes:
+    """SHA-1 digest of a byte string (plain C, FIPS 180-4)."""
+    a = _u8(x)
+    buf = a if a.size else np.zeros(1, np.uint8)
+    out = np.zeros(20, np.uint8)
+    dlib().dedup_ref_sha1(_ptr(buf), a.size, _ptr(out))
+    return out.tobytes()
+
+
+def fingerprints(x, chunk_size: int, n_threads: int | None = None) -> np.ndarray:
+    """fp[i] = SHA-1 of chunk i -> uint8[N, 20].  P:12 §2 "Hashing is the process of
+    calculating the hash value of each chunk"; §3.1(1) "SHA1, 20 bytes"."""
+    a = _u8(x)
+    if n_threads is None:
+        n_threads = len(os.sched_getaffinity(0))
+    N = (a.size + chunk_size - 1) // chunk_size
+    fp = np.zeros((max(1, N), 20), np.uint8)
+    buf = a if a.size else np.zeros(1, np.uint8)
+    st = dlib().dedup_ref_fingerprints(_ptr(buf), a.size, chunk_size, _ptr(fp), n_threads)
+    if st != 0:
+        raise ValueError(f"dedup_ref_fingerprints status {st}")
+    return fp[:N]
+
+
+def dedup_index(fps: np.ndarray, first_chunk: int = 0, seen: dict | None = None):
+    """Indexing step (§2 "Indexing is the process of comparing the hash value of
+    each chunk with the hash values of already stored chunks to determine whether it
+    is a duplicate"; §3.1(2) "the result of whether an index is hit or not
+    includes an index number and a hit/miss information pair").
+
+    Chunks are indexed in stream order; the index number of chunk i (global index
+    first_chunk + i) is the global index of the first chunk with the same
+    fingerprint (itself when it is new: a miss).  ``seen`` carries the index
+    across batches (fingerprint bytes -> first global index).
+    Returns (index uint64[N], hit uint8[N], seen)."""
+    if seen is None:
+        seen = {}
+    N = len(fps)
+    index = np.zeros(N, np.uint64)
+    hit = np.zeros(N, np.uint8)
+    for i in range(N):
+        key = bytes(fps[i])
+        g = first_chunk + i
+        if key in seen:
+            index[i] = seen[key]
+            hit[i] = 1
+        else:
+            seen[key] = g
+            index[i] = g
+    return index, hit, seen

@@ -18,7 +18,9 @@ HOST_LIB = os.path.join(_HERE, "libsynth.so")
 CUDA_LIB = os.path.join(_HERE, "libsynth_cuda.so")
 
 TEXT, RANDOM, ZERORUNS, MIX, CR2 = 0, 1, 2, 3, 4
-CLASSES = {"text": TEXT, "random": RANDOM, "zeroruns": ZERORUNS, "mix": MIX, "cr2": CR2}
+DEDUP = 0x10  # flag: dedup-2.0 logical stream over the base class (synth_core.h)
+CLASSES = {"text": TEXT, "random": RANDOM, "zeroruns": ZERORUNS, "mix": MIX, "cr2": CR2,
+           "mix_dedup": MIX | DEDUP}
 DEFAULT_SEED = 0x4C5A52
 
 NVCC_ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -65,6 +67,8 @@ def _hlib():
         L.syn_fill.argtypes = [ctypes.c_void_p, ctypes.c_size_t, ctypes.c_uint32, ctypes.c_int,
                                ctypes.c_uint64, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_int]
         L.syn_chunk_class_of.argtypes = [ctypes.c_int, ctypes.c_uint64, ctypes.c_uint64]
+        L.syn_dedup_source_of.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.syn_dedup_source_of.restype = ctypes.c_uint64
         _host = L
     return _host
 
@@ -76,6 +80,11 @@ def tables(seed: int = DEFAULT_SEED) -> np.ndarray:
         L.syn_build_tables(seed, ctypes.c_void_p(buf.ctypes.data))
         _tables_cache[seed] = buf
     return _tables_cache[seed]
+
+
+def dedup_source(chunk: int, seed: int = DEFAULT_SEED) -> int:
+    """Fresh chunk whose content logical chunk `chunk` of a dedup stream carries."""
+    return int(_hlib().syn_dedup_source_of(seed, chunk))
 
 
 def chunk_class(cls: int, chunk: int, seed: int = DEFAULT_SEED) -> int:

@@ -129,9 +129,33 @@ SYN_FN void syn_fill_text(uint8_t* out, uint32_t n, syn_rng* r, const syn_tables
   }
 }
 
+/* Dedup-2.0 logical stream (config 5; §4 "The deduplication and
+ * compression ratio are set to 2.0"): logical chunk i is fresh w.p. 1/2 (chunk
+ * 0 always); a duplicate copies the content of the nearest fresh chunk at or
+ * below a uniformly drawn earlier index r < i.  Content of a fresh chunk j = the
+ * base class's chunk j, so distinct fresh chunks differ (with overwhelming
+ * probability) and logical/unique ~ 2.0.  The flag SYN_DEDUP on the class
+ * selects this mapping. */
+#define SYN_DEDUP 0x10
+
+SYN_FN int syn_fresh(uint64_t seed, uint64_t i) {
+  return i == 0 || (syn_mix(seed ^ syn_mix(i ^ 0xDED0DED0ull)) & 1u);
+}
+
+SYN_FN uint64_t syn_dedup_source(uint64_t seed, uint64_t i) {
+  if (syn_fresh(seed, i)) return i;
+  uint64_t r = syn_mix(seed ^ syn_mix(i ^ 0x50C0CE5ull)) % i;
+  while (!syn_fresh(seed, r)) --r;
+  return r;
+}
+
 /* Generate chunk `chunk` (global index) of length n into out. */
 SYN_FN void syn_fill_chunk(uint8_t* out, uint32_t n, int cls, uint64_t seed, uint64_t chunk,
                            const syn_tables* t) {
+  if (cls & SYN_DEDUP) {
+    cls &= ~SYN_DEDUP;
+    chunk = syn_dedup_source(seed, chunk);
+  }
   int c = syn_chunk_class(cls, seed, chunk);
   syn_rng r = syn_chunk_rng(seed, chunk);
   if (c == SYN_TEXT) syn_fill_text(out, n, &r, t);

@@ -16,7 +16,7 @@ __global__ void syn_fill_kernel(uint8_t* out, size_t n, uint32_t C, int cls, uin
 extern "C" int syn_fill_device(void* d_out, size_t n, uint32_t chunk_size, int cls,
                                uint64_t seed, uint64_t first_chunk, const void* d_tables,
                                cudaStream_t stream) {
-  if (chunk_size == 0 || cls < 0 || cls >= SYN_NCLASS || (n && (!d_out || !d_tables))) return -1;
+  if (chunk_size == 0 || cls < 0 || (cls & ~SYN_DEDUP) >= SYN_NCLASS || (n && (!d_out || !d_tables))) return -1;
   size_t N = (n + chunk_size - 1) / chunk_size;
   if (N == 0) return 0;
   unsigned threads = 128;

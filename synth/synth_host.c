@@ -74,7 +74,7 @@ static void* syn_worker(void* a) {
 /* Fill out[0..n) with chunks first_chunk, first_chunk+1, ... of class cls. */
 int syn_fill(uint8_t* out, size_t n, uint32_t chunk_size, int cls, uint64_t seed,
              uint64_t first_chunk, const syn_tables* t, int n_threads) {
-  if (chunk_size == 0 || cls < 0 || cls >= SYN_NCLASS) return -1;
+  if (chunk_size == 0 || cls < 0 || (cls & ~SYN_DEDUP) >= SYN_NCLASS) return -1;
   syn_job j;
   memset(&j, 0, sizeof j);
   j.out = out; j.n = n; j.C = chunk_size; j.cls = cls; j.seed = seed; j.first = first_chunk;
@@ -92,3 +92,5 @@ int syn_fill(uint8_t* out, size_t n, uint32_t chunk_size, int cls, uint64_t seed
 int syn_chunk_class_of(int cls, uint64_t seed, uint64_t chunk) {
   return syn_chunk_class(cls, seed, chunk);
 }
+
+uint64_t syn_dedup_source_of(uint64_t seed, uint64_t chunk) { return syn_dedup_source(seed, chunk); }
