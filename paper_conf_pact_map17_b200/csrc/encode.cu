@@ -41,7 +41,6 @@ namespace {
 
 constexpr uint16_t kFirst = 0x8000;  // first entry of its bucket
 constexpr uint16_t kPos = 0x7FFF;
-constexpr uint32_t kMaxRuns = kMaxRunsL;  // runs of one byte value of length >= k, per chunk
 
 // ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K] during
 // the walk, reused as T[K], M[K] (token / match totals) after the chain phase
@@ -234,7 +233,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   const uint32_t kp = ld32u(data, p) & a.kmask;
   const bool prun = ((kp ^ (kp >> 8)) & (a.kmask >> 8)) == 0;  // key = one repeated byte
   const bool all_in_window = p <= a.W;
-  if (prun && all_in_window && nruns <= kMaxRuns)
+  if (prun && all_in_window && nruns <= a.L.max_runs)
     return best_match_runs(S, p, cap, kp, nruns, a, lane);
   // (generic path: window smaller than the prefix, many runs, or a plain key)
   uint32_t best = 0, blen = 0, rp = 0;
@@ -347,33 +346,37 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
 #ifdef LZR_PHASE_TIMING
     ++n_it;
 #endif
+    // one iteration = the literal stretch before the next candidate position
+    // q = p + L (from the candidate bitmap, up to 32 positions) and, if q was
+    // found, the token at q
     uint32_t bits = 0;
     if (p < P) bits = __funnelshift_r(S.cand[p >> 5], S.cand[(p >> 5) + 1], p & 31u);
-    uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
-    uint32_t tok_len = 0, r = 0;
-    if (L == 0) {  // candidate position: one token
+    const uint32_t L = bits ? (uint32_t)(__ffs(bits) - 1) : min(32u, n - p);
+    const uint32_t q = p + L;
+    uint32_t tok_len = 0, r = 0, cnt = L;  // cnt: token starts recorded, [p, p + cnt)
+    if (bits) {
 #ifdef LZR_PHASE_TIMING
       const long long tb0 = clock64();
 #endif
-      r = best_match(S, p, n, nruns, a, lane);
+      r = best_match(S, q, n, nruns, a, lane);
 #ifdef LZR_PHASE_TIMING
       t_bm += clock64() - tb0;
       ++n_bm;
 #endif
       const uint32_t l = r >> 16;
       tok_len = l >= a.m ? l : 1u;
-      L = 1;
+      cnt = L + 1;  // <= 32
     }
-    // record token starts [p, p+L) and (d-1) (lane 0 / lane 1, predicated)
+    // record token starts [p, p+cnt) and (d-1) at q (lane 0, predicated)
     {
       const uint32_t w = p >> 5, sh = p & 31u;
-      const uint32_t mask = L >= 32 ? 0xFFFFFFFFu : ((1u << L) - 1u);
+      const uint32_t mask = cnt >= 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
       red_or_if(lane == 0, &tbk[w], mask << sh);
-      red_or_if(lane == 0 && sh + L > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
-      st_u16_if(lane == 0 && tok_len > 1, d1 + p, 0xFFFFu - (r & 0xFFFFu));  // d - 1
+      red_or_if(lane == 0 && sh + cnt > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
+      st_u16_if(lane == 0 && tok_len > 1, d1 + q, 0xFFFFu - (r & 0xFFFFu));  // d - 1
     }
     // does this stretch meet the successor's parse?
-    if (K > 1 && k + 1 < K && p + L > nb) {
+    if (K > 1 && k + 1 < K && p + cnt > nb) {
       // one atomic read of the successor's progress, broadcast: per-lane reads
       // could see different values and split the warp (-> warp-sync deadlock)
       uint32_t pr = 0;
@@ -382,7 +385,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
         fence_acq_rel_cta();  // the successor's bits below pr are visible after this
       }
       pr = __shfl_sync(kFull, pr, 0);
-      const uint32_t lo = max(p, nb), hi = min(p + L, pr);
+      const uint32_t lo = max(p, nb), hi = min(p + cnt, pr);
       if (lo < hi) {
         uint32_t x = hi;
         for (uint32_t w = lo >> 5; w <= (hi - 1) >> 5; ++w) {
@@ -407,8 +410,9 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
         }
       }
     }
-    p += tok_len ? tok_len : L;
-    if (p - pub >= 64 || p >= n) {  // publish progress (a later publish only delays meeting)
+    p = bits ? q + tok_len : q;
+    // publish progress (a later publish only delays meeting; warp 0's is never read)
+    if (k > 0 && (p - pub >= 64 || p >= n)) {
       pub = p;
       if (lane == 0) {
         fence_acq_rel_cta();  // recorded token bits before the progress word
@@ -450,7 +454,7 @@ struct MaxThreads {
       K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : 1024)));
 };
 
-template <int K>
+template <int K, int NS>
 __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
@@ -468,9 +472,9 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
   S.cb = bms + nw;
   S.tb = bms + 2 * nw;
   S.runs = S.tb + K * a.L.tb_words;
-  S.ctrl = S.runs + kMaxRuns;
+  S.ctrl = S.runs + a.L.max_runs;
   S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
-  const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;
+  const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;  // NS == a.L.nsplit
   const uint32_t lt = lanemask_lt();
   const uint32_t tid = k * 32 + lane;
   // (d-1) of recorded matches: a per-group global scratch reused chunk after
@@ -503,6 +507,8 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     const uint32_t n = (uint32_t)min((size_t)a.C, a.n_bytes - lo);
     const uint8_t* src = a.in + lo;
     const uint32_t P = n >= a.m ? n - a.m + 1 : 0;  // positions that can start a match
+    // scatter split j covers positions [j*SS, (j+1)*SS) (SS a multiple of 32)
+    const uint32_t SS = align_up((P + NS - 1) / NS, 32);
     uint8_t* out = a.slots + (size_t)c * a.C;  // the chunk's workspace slot (its stream)
 
     // ---- a2: stage (TMA bulk for the 16-byte multiple, LDG for the tail); zero
@@ -514,9 +520,9 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     }
     for (uint32_t i = n16 + tid; i < n; i += nthr) S.data[i] = src[i];
     for (uint32_t i = n + tid; i < n + 20; i += nthr) S.data[i] = 0;
-    uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);    // B u16 counters
+    uint32_t* hist = reinterpret_cast<uint32_t*>(S.slot);    // NS x B u16 counters
     uint32_t* seen = reinterpret_cast<uint32_t*>(S.sorted);  // 2^fb-bit filter
-    for (uint32_t i = tid; i < B / 2; i += nthr) hist[i] = 0;
+    for (uint32_t i = tid; i < NS * B / 2; i += nthr) hist[i] = 0;
     for (uint32_t i = tid; i < (1u << (fb - 5)); i += nthr) seen[i] = 0;
     if (tid == 0) {
       S.ctrl[kCtrlU] = 0;
@@ -544,17 +550,18 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         const uint32_t key0 = __shfl_sync(kFull, key, 0);
         const bool uni = __all_sync(kFull, p < P && key == key0);
         const uint32_t h = khash(key, hb, a.kmask);
+        const uint32_t hs = (NS > 1 ? (p0 / SS) * B : 0u) + h;  // (split, bucket) counter
         const uint32_t gg = (key * 0x85EBCA6Bu) >> (32 - fb);
         if (uni) {
           uint32_t old = 0;
           if (lane == 0) {
-            atomicAdd(&hist[h >> 1], 32u << ((h & 1u) << 4));
+            atomicAdd(&hist[hs >> 1], 32u << ((hs & 1u) << 4));
             old = atomicOr(&seen[gg >> 5], 1u << (gg & 31u));
           }
           old = __shfl_sync(kFull, old, 0);
           dup = lane ? true : (old & (1u << (gg & 31u))) != 0;
         } else if (p < P) {
-          atomicAdd(&hist[h >> 1], 1u << ((h & 1u) << 4));
+          atomicAdd(&hist[hs >> 1], 1u << ((hs & 1u) << 4));
           dup = atomicOr(&seen[gg >> 5], 1u << (gg & 31u)) & (1u << (gg & 31u));
         }
         if (p < P)
@@ -566,7 +573,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
           if (lane == 0) b0 = atomicAdd(&S.ctrl[kCtrlRuns], (uint32_t)__popc(rb));
           b0 = __shfl_sync(kFull, b0, 0);
           const uint32_t idx = b0 + __popc(rb & lt);
-          if (rs && idx < kMaxRuns) S.runs[idx] = p;
+          if (rs && idx < a.L.max_runs) S.runs[idx] = p;
         }
       }
       if (lane == 0 && u) atomicAdd(&S.ctrl[kCtrlU], u);
@@ -578,23 +585,37 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     }
     const uint32_t nruns = S.ctrl[kCtrlRuns];
 
-    // ---- warp 0: exclusive scan of the B u16 counters (64 per round);
-    //      the other warps: zero the bitmaps, byte-change bitmap, walk state
+    // ---- warp 0: exclusive scan of the B bucket totals (2 buckets per lane and
+    //      round); split j's cursor of bucket h = start of h + counts of h in
+    //      splits < j.  The other warps: zero the bitmaps, byte-change bitmap,
+    //      walk state
     const uint32_t kk = K == 1 ? 0 : k - 1, KK = K == 1 ? 1 : K - 1;  // helper warp index
     if (k == 0) {
       uint32_t carry = 0;
       for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
         const bool act = w0 + lane < B / 2;
-        const uint32_t wv = act ? hist[w0 + lane] : 0;
-        const uint32_t c0 = wv & 0xFFFFu, sum = c0 + (wv >> 16);
+        uint32_t c0 = 0, c1 = 0;  // totals of buckets 2w, 2w+1
+        for (uint32_t j = 0; j < NS; ++j) {
+          const uint32_t wv = act ? hist[j * (B / 2) + w0 + lane] : 0;
+          c0 += wv & 0xFFFFu;
+          c1 += wv >> 16;
+        }
+        const uint32_t sum = c0 + c1;
         uint32_t incl = sum;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
           const uint32_t t = __shfl_up_sync(kFull, incl, o);
           if ((int)lane >= o) incl += t;
         }
-        const uint32_t excl = incl - sum + carry;
-        if (act) hist[w0 + lane] = (excl & 0xFFFFu) | ((excl + c0) << 16);
+        uint32_t e0 = incl - sum + carry, e1 = e0 + c0;  // running cursors
+        if (act) {
+          for (uint32_t j = 0; j < NS; ++j) {
+            const uint32_t wv = hist[j * (B / 2) + w0 + lane];
+            hist[j * (B / 2) + w0 + lane] = (e0 & 0xFFFFu) | (e1 << 16);
+            e0 += wv & 0xFFFFu;
+            e1 += wv >> 16;
+          }
+        }
         carry += __shfl_sync(kFull, incl, 31);
       }
     }
@@ -614,23 +635,25 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
     }
     GSYNC(3);
 
-    // ---- warp 0: stable scatter, 4 blocks of 32 positions per round so that the
-    //      MATCH.ANY latencies overlap; the other warps: run ends
-    if (k == 0) {
-      uint16_t* cur = S.slot;
-      for (uint32_t p0 = 0; p0 < P; p0 += 128) {
+    // ---- warps j < NS: stable scatter of split j (positions [j*SS, (j+1)*SS))
+    //      with its own cursors, 4 blocks of 32 positions per round so that the
+    //      MATCH.ANY latencies overlap; the last warp then: run ends
+    if (k < NS) {
+      uint16_t* cur = S.slot + k * B;
+      const uint32_t pe = min(P, (k + 1) * SS);
+      for (uint32_t p0 = k * SS; p0 < pe; p0 += 128) {
         uint32_t h[4], peers[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const uint32_t p = p0 + 32 * u + lane;
-          h[u] = p < P ? khash(ld32u(S.data, p) & a.kmask, hb, a.kmask) : 0xFFFFFFFFu;
+          h[u] = p < pe ? khash(ld32u(S.data, p) & a.kmask, hb, a.kmask) : 0xFFFFFFFFu;
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const uint32_t p = p0 + 32 * u + lane;
-          const bool act = p < P;
+          const bool act = p < pe;
           const uint32_t basev = act ? cur[h[u]] : 0;
           if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)p;
           __syncwarp();
@@ -639,18 +662,22 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
         }
       }
     }
-    if (K == 1 || k != 0) {
-      for (uint32_t j = kk * 32 + lane; j < min(nruns, kMaxRuns); j += KK * 32) {
+    if (k == K - 1) {
+      for (uint32_t j = lane; j < min(nruns, a.L.max_runs); j += 32) {
         const uint32_t st = S.runs[j];
         S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
       }
     }
     GSYNC(4);
 
-    // ---- mark the first entry of every non-empty bucket (cur[h] = end of h)
-    for (uint32_t hh = tid; hh < B; hh += nthr) {
-      const uint32_t st = hh ? S.slot[hh - 1] : 0u;
-      if (S.slot[hh] > st) S.sorted[st] |= kFirst;
+    // ---- mark the first entry of every non-empty bucket (the last split's
+    //      cursor of h = end of h)
+    {
+      const uint16_t* endc = S.slot + (NS - 1) * B;
+      for (uint32_t hh = tid; hh < B; hh += nthr) {
+        const uint32_t st = hh ? endc[hh - 1] : 0u;
+        if (endc[hh] > st) S.sorted[st] |= kFirst;
+      }
     }
     GSYNC(5);
 
@@ -841,7 +868,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
   }
 }
 
-template <int K>
+template <int K, int NS>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
   const int max_groups = MaxThreads<K>::value / (32 * K);
@@ -849,12 +876,12 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   if (groups > 15) groups = 15;  // named barriers 1..15
   if (groups < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)groups * a.L.per_group;
-  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K>,
+  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t grid = need < (uint32_t)sm_count ? need : (uint32_t)sm_count;
-  lzr_encode_kernel<K><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -872,11 +899,24 @@ extern "C" int lzr_debug_phase_times(unsigned long long* out) {
 cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s,
                           int* launches) {
   switch (a.L.K) {
-    case 1: return launch_k<1>(a, sm_count, smem_optin, s, launches);
-    case 2: return launch_k<2>(a, sm_count, smem_optin, s, launches);
-    case 3: return launch_k<3>(a, sm_count, smem_optin, s, launches);
-    case 4: return launch_k<4>(a, sm_count, smem_optin, s, launches);
-    case 8: return launch_k<8>(a, sm_count, smem_optin, s, launches);
+    case 1: return launch_k<1, 1>(a, sm_count, smem_optin, s, launches);
+    case 2: return launch_k<2, 1>(a, sm_count, smem_optin, s, launches);
+    case 3: return launch_k<3, 1>(a, sm_count, smem_optin, s, launches);
+    case 4:
+      switch (a.L.nsplit) {
+        case 1: return launch_k<4, 1>(a, sm_count, smem_optin, s, launches);
+        case 2: return launch_k<4, 2>(a, sm_count, smem_optin, s, launches);
+        case 4: return launch_k<4, 4>(a, sm_count, smem_optin, s, launches);
+        default: return cudaErrorInvalidConfiguration;
+      }
+    case 8:
+      switch (a.L.nsplit) {
+        case 1: return launch_k<8, 1>(a, sm_count, smem_optin, s, launches);
+        case 2: return launch_k<8, 2>(a, sm_count, smem_optin, s, launches);
+        case 4: return launch_k<8, 4>(a, sm_count, smem_optin, s, launches);
+        case 8: return launch_k<8, 8>(a, sm_count, smem_optin, s, launches);
+        default: return cudaErrorInvalidConfiguration;
+      }
     default: return cudaErrorInvalidConfiguration;
   }
 }

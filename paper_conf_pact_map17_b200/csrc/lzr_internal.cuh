@@ -85,10 +85,15 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
 }
 
 // ---- encode kernel shared-memory layout (one region per group of K warps) ---
-constexpr uint32_t kMaxRunsL = 24;  // run list entries per chunk (encode.cu kMaxRuns)
+// run list capacity per chunk (runs of one byte value of length >= k): about
+// one zero run per 128 bytes of chunk (the zero-runs class has one per ~300 B)
+__host__ __device__ inline uint32_t enc_max_runs(uint32_t C) {
+  const uint32_t r = (C / 128 + 7) & ~7u;
+  return r < 24 ? 24 : r;
+}
 
 struct EncLayout {
-  uint32_t K, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, tb_words, fbits;
+  uint32_t K, nsplit, max_runs, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, tb_words, fbits;
 };
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
@@ -97,12 +102,20 @@ __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
   return hb;
 }
 
-__host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K) {
+// K warps per chunk; NS of them share the index scatter, each with its own
+// cursor array, so NS * B u16 counters must fit the 2 max(C, B)-byte slot
+// region: B = (largest power of two <= C) / NS
+__host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t NS) {
   EncLayout L;
   L.K = K;
   L.hbits = enc_hash_bits(C);
-  L.fbits = 5;  // raw pre-filter: 2^fbits bits inside the 2C-byte index region, <= 2^15
-  while ((2u << L.fbits) <= 16 * C && L.fbits < 15) ++L.fbits;
+  L.nsplit = 1;
+  while (L.nsplit < NS && L.hbits > 4) {
+    --L.hbits;
+    L.nsplit <<= 1;
+  }
+  L.fbits = 5;  // raw pre-filter: 2^fbits bits inside the 2C-byte index region (16C bits)
+  while ((2u << L.fbits) <= 16 * C && L.fbits < 20) ++L.fbits;
   uint32_t B = 1u << L.hbits;
   // chunk bytes + 20 zero bytes: 16-byte compares read up to 19 bytes past n
   uint32_t o = align_up(C + 20, 4);
@@ -114,7 +127,8 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K) {
   L.bm_words = (C + 31) / 32 + 1;  // candidate / byte-change: +1 for two-word funnel reads
   L.tb_words = (C + 31) / 32;      // per-segment token-start bitmaps
   // candidate, byte-change, K token-start bitmaps; run list; ctrl (4 + 2K words)
-  o += 4 * (2 * L.bm_words + K * L.tb_words + kMaxRunsL + 4 + 2 * K);
+  L.max_runs = enc_max_runs(C);
+  o += 4 * (2 * L.bm_words + K * L.tb_words + L.max_runs + 4 + 2 * K);
   o = align_up(o, 8);
   L.off_mbar = o;
   o += 8;
@@ -155,5 +169,16 @@ cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const 
 cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,
                           size_t n_bytes, uint32_t C, uint32_t m, uint8_t* out, int32_t* err,
                           int sm_count, int smem_optin, cudaStream_t s, int* launches);
+
+// dedup.cu
+cudaError_t launch_sha1(const uint8_t* in, size_t n, uint32_t C, uint8_t* fp, cudaStream_t s,
+                        int* launches);
+size_t dedup_entry_bytes();
+cudaError_t launch_index(const uint8_t* fps, size_t N, uint64_t first, void* table, uint32_t n_bins,
+                         uint32_t bin_slots, uint64_t* index, uint32_t* unique, uint32_t* overflow,
+                         cudaStream_t s, int* launches);
+cudaError_t launch_gather(const uint8_t* in, size_t n, uint32_t C, const uint32_t* unique,
+                          const uint64_t* rank, uint8_t* out, int sm_count, cudaStream_t s,
+                          int* launches);
 
 }  // namespace lzr
