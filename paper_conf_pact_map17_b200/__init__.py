@@ -18,6 +18,7 @@ __all__ = [
     "Params", "LzrError", "lib", "num_chunks", "compress_bound", "compress_workspace_bytes",
     "compress", "compress_encode", "compress_compact", "scan_sizes", "decompress",
     "compress_host", "validate_params", "status_str", "last_launch_count",
+    "fingerprint", "DedupIndex", "gather_chunks", "dedup_compress",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -31,7 +32,8 @@ EXPORTED_SYMBOLS = [
     "lzr_compress_chunks", "lzr_compress_encode", "lzr_compress_compact",
     "lzr_scan_workspace_bytes", "lzr_scan_sizes", "lzr_decompress_chunks",
     "lzr_compress_host_scratch_bytes", "lzr_compress_host", "lzr_status_str",
-    "lzr_last_launch_count",
+    "lzr_last_launch_count", "lzr_fingerprint_chunks", "lzr_dedup_table_bytes", "lzr_dedup_index",
+    "lzr_gather_chunks",
 ]
 
 
@@ -96,6 +98,12 @@ def lib():
         L.lzr_status_str.argtypes = [ctypes.c_int]
         L.lzr_status_str.restype = ctypes.c_char_p
         L.lzr_last_launch_count.argtypes = []
+        L.lzr_fingerprint_chunks.argtypes = [vp, sz, ctypes.c_uint32, vp, vp]
+        L.lzr_dedup_table_bytes.argtypes = [ctypes.c_uint32, ctypes.c_uint32]
+        L.lzr_dedup_table_bytes.restype = sz
+        L.lzr_dedup_index.argtypes = [vp, sz, u64, vp, ctypes.c_uint32, ctypes.c_uint32, vp, vp, vp,
+                                      vp]
+        L.lzr_gather_chunks.argtypes = [vp, sz, ctypes.c_uint32, vp, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -262,3 +270,97 @@ def compress_host(h_in, p: Params = Params(), batch_bytes: int = 0, scratch=None
         ctypes.byref(tot), batch_bytes, _ptr(scratch), scratch.numel())
     _check(st, "lzr_compress_host")
     return h_out, h_sizes[:N], h_offsets[:N], tot.value
+
+
+# ---- dedup upstream of compression (include/lzr.h) ---------------
+def fingerprint(t, chunk_size: int = 4096, out=None, stream=None):
+    """SHA-1 of every chunk of a uint8 CUDA tensor -> uint8[N, 20] CUDA tensor."""
+    import torch
+
+    _require_cuda_u8(t, "input")
+    n = t.numel()
+    N = -(-n // chunk_size)
+    if out is None:
+        out = torch.empty((max(1, N), 20), dtype=torch.uint8, device=t.device)
+    st = lib().lzr_fingerprint_chunks(_ptr(t), n, chunk_size, _ptr(out), _stream(stream, t.device))
+    _check(st, "lzr_fingerprint_chunks")
+    return out[:N]
+
+
+class DedupIndex:
+    """Bin-partitioned fingerprint index kept on the device across batches
+    (n_bins bins x bin_slots entries; zero-filled = empty)."""
+
+    def __init__(self, n_bins: int, bin_slots: int, device=None):
+        import torch
+
+        self.n_bins, self.bin_slots = n_bins, bin_slots
+        dev = torch.device(device) if device is not None else torch.device("cuda")
+        nb = lib().lzr_dedup_table_bytes(n_bins, bin_slots)
+        self.table = torch.zeros(max(256, nb), dtype=torch.uint8, device=dev)
+        self.overflow = torch.zeros(1, dtype=torch.int32, device=dev)
+
+    @classmethod
+    def for_chunks(cls, n_chunks: int, device=None, bin_slots: int = 64):
+        """Sized for n_chunks fingerprints at <= 50% load."""
+        n_bins = max(1, -(-2 * max(1, n_chunks) // bin_slots))
+        return cls(n_bins, bin_slots, device)
+
+    def reset(self):
+        self.table.zero_()
+        self.overflow.zero_()
+
+    def index(self, fp, first_chunk: int = 0, index=None, unique=None, stream=None):
+        """-> (index int64[N]: first global index with the same fingerprint,
+        unique int32[N]: 1 on a miss).  Nothing is synchronised."""
+        import torch
+
+        N = fp.shape[0]
+        dev = fp.device
+        if index is None:
+            index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+        if unique is None:
+            unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+        st = lib().lzr_dedup_index(_ptr(fp), N, first_chunk, _ptr(self.table), self.n_bins,
+                                   self.bin_slots, _ptr(index), _ptr(unique), _ptr(self.overflow),
+                                   _stream(stream, dev))
+        _check(st, "lzr_dedup_index")
+        return index[:N], unique[:N]
+
+
+def gather_chunks(t, chunk_size: int, unique, rank, out, stream=None):
+    """Copy the unique chunks of t to out in stream order (out + rank[i] * C)."""
+    st = lib().lzr_gather_chunks(_ptr(t), t.numel(), chunk_size, _ptr(unique), _ptr(rank), _ptr(out),
+                                 _stream(stream, t.device))
+    _check(st, "lzr_gather_chunks")
+    return out
+
+
+def dedup_compress(t, p: Params = Params(), index: DedupIndex | None = None, first_chunk: int = 0,
+                   ws: Workspace | None = None, stream=None):
+    """Dedup before compression (§3.3): fingerprint every chunk, index the
+    fingerprints, gather the unique chunks, compress them.  Synchronises once to
+    size the unique buffer.  Returns a dict with fp, index, unique, rank,
+    n_unique, the gathered unique bytes and compress()'s (out, sizes, offsets,
+    total) over them."""
+    import torch
+
+    C = p.chunk_size
+    if index is None:
+        index = DedupIndex.for_chunks(-(-t.numel() // C), t.device)
+    fp = fingerprint(t, C, stream=stream)
+    idx, uniq = index.index(fp, first_chunk, stream=stream)
+    rank, n_uniq_t = scan_sizes(uniq, stream=stream)
+    n = t.numel()
+    N = fp.shape[0]
+    nu = int(n_uniq_t.item())
+    last_unique = N > 0 and bool(uniq[N - 1].item())
+    ubytes = nu * C
+    if last_unique and n % C:
+        ubytes -= C - n % C  # the short tail chunk is the last unique one
+    ubuf = torch.empty(max(1, ubytes), dtype=torch.uint8, device=t.device)
+    gather_chunks(t, C, uniq, rank, ubuf, stream=stream)
+    u = ubuf[:ubytes]
+    out, sizes, offs, total = compress(u, p, ws=ws, stream=stream)
+    return {"fp": fp, "index": idx, "unique": uniq, "rank": rank, "n_unique": nu, "unique_bytes": u,
+            "out": out, "sizes": sizes, "offsets": offs, "total": total}

@@ -57,6 +57,20 @@ uint32_t enc_warps_per_chunk(uint32_t C) {
   return C > 4096 ? 8u : (C >= 1024 ? 4u : 1u);
 }
 
+// warps that share the index scatter (each a contiguous position range with
+// its own cursor array; the hash table shrinks by the same factor)
+uint32_t enc_scatter_splits(uint32_t K) {
+  static int env = -1;
+  if (env < 0) {
+    const char* e = getenv("LZR_ENCODE_SPLITS");
+    env = (e && (*e == '1' || *e == '2' || *e == '4' || *e == '8')) ? (*e - '0') : 0;
+  }
+  // default (config-3 sweep, 1 x B200): 1 split at K = 4 (C = 4 KiB: the full
+  // C-bucket table matters more than the serial scatter), 4 at K = 8
+  const uint32_t ns = env > 0 ? (uint32_t)env : (K >= 8 ? 4u : 1u);
+  return K < 4 ? 1u : (ns < K ? ns : K);  // (kernels are instantiated for these)
+}
+
 }  // namespace
 
 WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
@@ -149,7 +163,8 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.M = p->max_match;
   a.kbytes = p->min_match < 4 ? p->min_match : 4;
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
-  a.L = enc_layout(p->chunk_size, enc_warps_per_chunk(p->chunk_size));
+  const uint32_t K = enc_warps_per_chunk(p->chunk_size);
+  a.L = enc_layout(p->chunk_size, K, enc_scatter_splits(K));
   // positions are 15-bit in the index (bit 15 marks bucket starts) and one
   // chunk's index must fit one CTA's shared memory
   if (p->chunk_size > 32768 || (int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;
@@ -235,6 +250,52 @@ int lzr_scan_sizes(const uint32_t* d_sizes, size_t n, uint64_t base, uint64_t* d
   if (workspace_bytes < scan_ws_bytes(n)) return LZR_ERR_CAPACITY;
   if (launch_scan(d_sizes, n, base, nullptr, d_offsets, d_total, d_workspace, s, &t_launches) !=
       cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_fingerprint_chunks(const void* d_in, size_t n_bytes, uint32_t chunk_size, uint8_t* d_fp,
+                           lzr_stream_t stream) {
+  t_launches = 0;
+  if (n_bytes == 0) return LZR_OK;
+  if (!d_in || !d_fp || chunk_size == 0) return LZR_ERR_INVALID_ARG;
+  if (launch_sha1((const uint8_t*)d_in, n_bytes, chunk_size, d_fp, (cudaStream_t)stream,
+                  &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+size_t lzr_dedup_table_bytes(uint32_t n_bins, uint32_t bin_slots) {
+  return (size_t)n_bins * bin_slots * dedup_entry_bytes();
+}
+
+int lzr_dedup_index(const uint8_t* d_fp, size_t n_chunks, uint64_t first_chunk, void* d_table,
+                    uint32_t n_bins, uint32_t bin_slots, uint64_t* d_index, uint32_t* d_unique,
+                    uint32_t* d_overflow, lzr_stream_t stream) {
+  t_launches = 0;
+  if (n_chunks == 0) return LZR_OK;
+  if (!d_fp || !d_table || !d_index || !d_unique || !d_overflow || n_bins == 0 || bin_slots == 0)
+    return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_table, 256) || !aligned(d_index, 8) || !aligned(d_unique, 4) ||
+      !aligned(d_overflow, 4))
+    return LZR_ERR_INVALID_ARG;
+  if (launch_index(d_fp, n_chunks, first_chunk, d_table, n_bins, bin_slots, d_index, d_unique,
+                   d_overflow, (cudaStream_t)stream, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_gather_chunks(const void* d_in, size_t n_bytes, uint32_t chunk_size,
+                      const uint32_t* d_unique, const uint64_t* d_rank, void* d_out,
+                      lzr_stream_t stream) {
+  t_launches = 0;
+  if (n_bytes == 0) return LZR_OK;
+  if (!d_in || !d_unique || !d_rank || !d_out || chunk_size == 0) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_unique, 4) || !aligned(d_rank, 8)) return LZR_ERR_INVALID_ARG;
+  DevInfo di;
+  if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
+  if (launch_gather((const uint8_t*)d_in, n_bytes, chunk_size, d_unique, d_rank, (uint8_t*)d_out,
+                    di.sm_count, (cudaStream_t)stream, &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;
 }
