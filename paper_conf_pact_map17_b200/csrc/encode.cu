@@ -444,18 +444,35 @@ __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
   return n >= base + 32 ? 0xFFFFFFFFu : (n > base ? (1u << (n - base)) - 1u : 0u);
 }
 
-// threads per CTA at most: 10 groups of 1 or 2 warps, 9 of 3, 8 of 4
+// threads per CTA at most (K = 1..3: 10 groups of 1 or 2 warps, 9 of 3)
+// CTA shapes (A/B on 1 x B200, tools/ab.sh): K = 4 runs 3 CTAs of 3 groups per
+// SM (9 groups = 36 warps at <= 56 registers; 1 CTA of 8 groups: mix 46.9 ->
+// 50.1 GB/s, zero-runs 61.7 -> 71.7); K = 8 (C > 4 KiB) see LZR_K8_*.
 #ifndef LZR_K4_THREADS
-#define LZR_K4_THREADS 1024
+#define LZR_K4_THREADS 384
+#endif
+#ifndef LZR_K4_MINB
+#define LZR_K4_MINB 3
+#endif
+#ifndef LZR_K8_THREADS
+#define LZR_K8_THREADS 1024
+#endif
+#ifndef LZR_K8_MINB
+#define LZR_K8_MINB 1
 #endif
 template <int K>
 struct MaxThreads {
   static constexpr int value =
-      K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : 1024)));
+      K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : LZR_K8_THREADS)));
+};
+template <int K>
+struct MinBlocks {
+  static constexpr int value = K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1);
 };
 
 template <int K, int NS>
-__global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(const EncArgs a) {
+__global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
+    lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
   const uint32_t warp = threadIdx.x >> 5;
@@ -637,7 +654,9 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, 1) lzr_encode_kernel(con
 
     // ---- warps j < NS: stable scatter of split j (positions [j*SS, (j+1)*SS))
     //      with its own cursors, 4 blocks of 32 positions per round so that the
-    //      MATCH.ANY latencies overlap; the last warp then: run ends
+    //      MATCH.ANY latencies overlap; the last warp then: run ends.  (A
+    //      bucket-partitioned variant -- every warp scans all positions and
+    //      scatters its own buckets -- measured slower: 50.1 -> 44.6 GB/s mix.)
     if (k < NS) {
       uint16_t* cur = S.slot + k * B;
       const uint32_t pe = min(P, (k + 1) * SS);
@@ -879,8 +898,16 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
+  // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
+  int per_sm = 1;
+  if (MinBlocks<K>::value > 1 &&
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS>,
+                                                    groups * 32 * K, smem) != cudaSuccess)
+    per_sm = 1;
+  if (per_sm < 1) per_sm = 1;
   const uint32_t need = (a.N + groups - 1) / groups;
-  const uint32_t grid = need < (uint32_t)sm_count ? need : (uint32_t)sm_count;
+  const uint32_t cap = (uint32_t)(sm_count * per_sm);
+  const uint32_t grid = need < cap ? need : cap;
   lzr_encode_kernel<K, NS><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
