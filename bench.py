@@ -131,16 +131,36 @@ class ClockSampler:
                 "samples": len(self.sm), "source": "NVML, 10 ms period, timed region only"}
 
 
-def traffic_from_profiles(workload: str):
-    """dram read+write bytes per encode launch from the committed ncu summary."""
+def _profile_entry(workload: str):
     path = os.path.join(ROOT, "profiles", "encode_ncu_summary.json")
     try:
         with open(path) as f:
-            d = json.load(f)
-        e = d.get(workload)
-        return float(e["dram_bytes_per_launch"]) if e else None
+            return json.load(f).get(workload)
     except Exception:
         return None
+
+
+def traffic_from_profiles(workload: str):
+    """dram read+write bytes per encode launch from the committed ncu summary."""
+    e = _profile_entry(workload)
+    return float(e["dram_bytes_per_launch"]) if e else None
+
+
+def issue_limiter(workload: str, enc_avg_s: float, sm_mhz, n_sms: int):
+    """The encode kernel's real limiter: warp-instruction issue.  Warp
+    instructions per launch from the committed ncu capture of the same workload
+    (profiles/encode_ncu_summary.json), divided by the live average launch time,
+    against the issue peak 4 warp-instructions / cycle / SM (one per SMSP) x SMs
+    x the SM clock sampled during the timed region."""
+    e = _profile_entry(workload)
+    if not e or not e.get("warp_inst_per_launch") or not sm_mhz:
+        return None
+    inst = float(e["warp_inst_per_launch"])
+    achieved = inst / enc_avg_s / 1e9
+    peak = 4 * n_sms * float(sm_mhz) * 1e6 / 1e9
+    return {"kind": "issue", "achieved": round(achieved, 2), "peak": round(peak, 2),
+            "unit": "G warp-inst/s", "frac": round(achieved / peak, 4),
+            "warp_inst_per_launch": inst, "source": e.get("source")}
 
 
 def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
@@ -496,6 +516,10 @@ def main():
         "clocks": clk.summary(),
         "gpu_launches": launches[0],
     }
+    lim = issue_limiter(workload, enc_avg_s, line["clocks"].get("sm_mhz"),
+                        torch.cuda.get_device_properties(dev).multi_processor_count)
+    if lim:
+        line["roofline"]["limiter"] = lim
 
     # ---- decompression of the same batch, output GB/s
     if not a.no_decode:

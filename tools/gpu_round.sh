@@ -1,0 +1,11 @@
+# full round check: gpu tests, smoke, default bench, reference arm, config-3/5 lines, ncu launch list + encode capture
+R=${1:-r01c}
+mkdir -p gpurun_out
+timeout 1200 python -m pytest tests -m gpu -q 2>&1 | tail -n 3 > gpurun_out/pytest_gpu_$R.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_$R.log 2>&1
+timeout 600 python bench.py > gpurun_out/bench_default_$R.log 2>&1
+timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref_$R.log 2>&1
+for C in 8192 16384 32768; do timeout 600 python bench.py --config 3 --chunk-size $C --steps 3 --no-cpu --no-e2e > gpurun_out/bench_cfg3_${C}_$R.log 2>&1; done
+timeout 900 python bench.py --config 5 --steps 5 > gpurun_out/bench_cfg5_$R.log 2>&1
+bash tools/ncu_bench.sh $R
+tail -n 3 gpurun_out/pytest_gpu_$R.log gpurun_out/smoke_$R.log

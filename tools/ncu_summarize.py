@@ -51,6 +51,8 @@ summ_path = os.path.join(ROOT, "profiles", "encode_ncu_summary.json")
 summ = json.load(open(summ_path)) if os.path.exists(summ_path) else {}
 summ[workload] = {"round": R, "dram_bytes_per_launch": full["dram_bytes_per_launch"],
                   "duration_s": full.get("gpu__time_duration.sum"),
+                  "warp_inst_per_launch": full.get("smsp__inst_executed.sum"),
+                  "ipc": full.get("sm__inst_executed.avg.per_cycle_active"),
                   "source": f"profiles/ncu_{R}.json (ncu --set full, one encode launch of bench.py)"}
 json.dump(summ, open(summ_path, "w"), indent=1)
 json.dump(out, open(os.path.join(ROOT, "profiles", f"ncu_{R}.json"), "w"), indent=1)
