@@ -243,16 +243,18 @@ def decompress(comp, sizes, offsets, n: int, p: Params = Params(), out=None, err
     return out[:n], error
 
 
-def compress_host(h_in, p: Params = Params(), batch_bytes: int = 0, scratch=None, h_out=None,
-                  h_sizes=None, h_offsets=None):
+def compress_host(h_in, p: Params = Params(), batch_bytes: int = 16 << 20, scratch=None,
+                  h_out=None, h_sizes=None, h_offsets=None):
     """End-to-end compression of a host (preferably pinned) uint8 tensor through
-    the C ABI's host-buffer pipeline (H2D, kernels, D2H inside).  Synchronous.
+    the C ABI's host-buffer pipeline (H2D, kernels, D2H inside; 16 MiB batches
+    by default, 0 = one batch).  Synchronous.
     Returns (h_out, h_sizes, h_offsets, total) on the host."""
     import torch
 
     n = h_in.numel()
     N = num_chunks(n, p)
-    if batch_bytes == 0:
+    batch_bytes = -(-batch_bytes // p.chunk_size) * p.chunk_size
+    if batch_bytes == 0 or batch_bytes > n:
         batch_bytes = max(p.chunk_size, -(-n // p.chunk_size) * p.chunk_size)
     need = lib().lzr_compress_host_scratch_bytes(batch_bytes, ctypes.byref(p.c()))
     if scratch is None or scratch.numel() < need:

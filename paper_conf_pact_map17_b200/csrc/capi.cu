@@ -354,14 +354,25 @@ HostSet carve(uint8_t* base, size_t batch, const lzr_params* p) {
 }
 }  // namespace
 
-// Three buffer sets on three streams: while batch b computes, batch b-1's
-// compressed bytes go back (D2H) and batch b+1's input comes in (H2D); a set is
-// reused only after its D2H was issued on its own stream (stream order).
-constexpr int kHostSets = 3;
+// host_sets() buffer sets on as many streams: while batch b computes, earlier
+// batches' compressed bytes go back (D2H) and later batches' inputs come in
+// (H2D); a set is reused only after its D2H was issued on its own stream
+// (stream order).
+constexpr int kMaxHostSets = 8;
+// default 4 sets (e2e sweep on 1 x B200, 256 MiB mix, PCIe 55 GB/s one way / 94
+// both ways: 3 sets x 32 MiB 31.1 GB/s, 4 x 16 MiB 35.7, 6 x 16 MiB 32.6)
+int host_sets() {  // LZR_HOST_SETS=2..8 overrides (tuning)
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("LZR_HOST_SETS");
+    v = (e && *e >= '2' && *e <= '8') ? (*e - '0') : 4;
+  }
+  return v;
+}
 
 size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
   if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
-  return kHostSets * align_up_z(set_bytes(batch_bytes, p), 256);
+  return host_sets() * align_up_z(set_bytes(batch_bytes, p), 256);
 }
 
 int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, void* h_out,
@@ -381,9 +392,10 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   if (batch_bytes % C) return LZR_ERR_INVALID_ARG;
   if (!aligned(d_scratch, 256)) return LZR_ERR_INVALID_ARG;
   const size_t per = align_up_z(set_bytes(batch_bytes, p), 256);
+  const int kHostSets = host_sets();
   if (scratch_bytes < kHostSets * per) return LZR_ERR_CAPACITY;
-  HostSet set[kHostSets];
-  cudaStream_t s[kHostSets];
+  HostSet set[kMaxHostSets];
+  cudaStream_t s[kMaxHostSets];
   int made = 0;
   for (; made < kHostSets; ++made) {
     set[made] = carve((uint8_t*)d_scratch + made * per, batch_bytes, p);
