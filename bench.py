@@ -47,8 +47,8 @@ def parse():
     ap.add_argument("--cls", default="mix")
     ap.add_argument("--config", type=int, default=2, choices=[1, 2, 3, 4, 5],
                     help="BASELINE.json config: 1 = 1 MiB, 2 = 256 MiB/GPU (default), 3 = 1 GiB/GPU "
-                         "(with --chunk-size), 4 = 16 GiB sharded, 5 = 8 GiB unique of a 16 GiB "
-                         "dedup-2.0 stream, sharded")
+                         "(with --chunk-size), 4 = 16 GiB sharded, 5 = 16 GiB logical dedup-2.0 "
+                         "stream: GPU dedup (global index over ranks) then compress the unique chunks")
     ap.add_argument("--bytes-per-rank", type=int, default=None)
     ap.add_argument("--chunk-size", type=int, default=CHUNK)
     ap.add_argument("--cpu-sample-bytes", type=int, default=24 << 20)
@@ -227,50 +227,75 @@ def run_reference(a):
     print(json.dumps(line), flush=True)
 
 
-def run_dedup_single(a):
-    """Config 5 on one GPU: the integrated dedup-before-compression step
-    (§3.3).  One step over the 16 GiB logical
-    dedup-2.0 stream: reset the index, SHA-1 every chunk, index (first
-    occurrence), scan the unique flags, gather the unique chunks, compress them
-    (encode + scan/compaction).  value = unique (compressor input) bytes per
-    second; logical_value = logical stream bytes per second."""
+def run_dedup(a):
+    """Config 5: the integrated dedup-before-compression step (P:16 §3.3;
+    SURVEY.md §8(f) N2) over the 16 GiB logical dedup-2.0 stream.  One step:
+    reset the index, SHA-1 every chunk, index (first occurrence in stream
+    order), scan the unique flags, gather the unique chunks, compress them
+    (encode + scan/compaction).  Under torchrun every rank owns a contiguous
+    chunk range of the logical stream and the index is global (ShardedDedup:
+    NCCL all-to-all of fingerprint records to their owner rank and of the index
+    numbers back), then an all-gather of the per-rank compressed totals.
+    value = unique (compressor input) bytes per second over all ranks;
+    logical_value = logical stream bytes per second."""
     import numpy as np
     import torch
+    import torch.distributed as dist
 
     import synth
     import paper_conf_pact_map17_b200 as lzr
+    from paper_conf_pact_map17_b200.dist import ShardedDedup, shard_range
 
-    dev = torch.device("cuda", 0)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    grank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
+    sharded = "WORLD_SIZE" in os.environ and "MASTER_ADDR" in os.environ
+    if sharded:
+        dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
     p = lzr.Params(chunk_size=C)
-    n = ((a.bytes_per_rank or (16 << 30)) // C) * C
-    N = n // C
+    n_glob = ((a.bytes_per_rank * world if a.bytes_per_rank else (16 << 30)) // C) * C
+    N_glob = n_glob // C
+    lo, hi = shard_range(N_glob, world, grank) if sharded else (0, N_glob)
+    n = (hi - lo) * C
+    N = hi - lo
     stream = torch.cuda.current_stream(dev)
     x = torch.empty(n, dtype=torch.uint8, device=dev)
-    synth.fill_device(x, C, "mix_dedup")
+    synth.fill_device(x, C, "mix_dedup", first_chunk=lo)
     fp = torch.empty((N, 20), dtype=torch.uint8, device=dev)
-    index = lzr.DedupIndex.for_chunks(N, dev)
     idx = torch.empty(N, dtype=torch.int64, device=dev)
     uniq = torch.empty(N, dtype=torch.int32, device=dev)
-    rank = torch.empty(N, dtype=torch.int64, device=dev)
+    if sharded:
+        sd = ShardedDedup(N, device=dev)
+        index = sd.ops.index
+    else:
+        index = lzr.DedupIndex.for_chunks(N, dev)
+    rank_ = torch.empty(N, dtype=torch.int64, device=dev)
     nu_t = torch.zeros(1, dtype=torch.int64, device=dev)
     scan_ws = torch.empty(max(256, lzr.lib().lzr_scan_workspace_bytes(N)), dtype=torch.uint8, device=dev)
+    totals_all = torch.zeros(world, dtype=torch.int64, device=dev)
     launches = [0]
 
     def dedup_part():
+        nonlocal idx, uniq
         index.reset()
-        lzr.fingerprint(x, C, out=fp)
-        launches[0] += lzr.last_launch_count()
-        index.index(fp, 0, index=idx, unique=uniq)
-        launches[0] += lzr.last_launch_count()
-        lzr.scan_sizes(uniq, 0, offsets=rank, total=nu_t, ws=scan_ws)
+        if sharded:
+            _, idx, uniq = sd(x, C, lo)
+            launches[0] += 6  # fingerprint, owner counts, route, insert, lookup, unroute
+        else:
+            lzr.fingerprint(x, C, out=fp)
+            launches[0] += lzr.last_launch_count()
+            index.index(fp, 0, index=idx, unique=uniq)
+            launches[0] += lzr.last_launch_count()
+        lzr.scan_sizes(uniq, 0, offsets=rank_, total=nu_t, ws=scan_ws)
         launches[0] += lzr.last_launch_count()
         return int(nu_t.item())  # host needs the unique count to size the compression
 
     nu = dedup_part()
     nub = nu * C
-    ubuf = torch.empty(nub, dtype=torch.uint8, device=dev)
+    ubuf = torch.empty(max(1, nub), dtype=torch.uint8, device=dev)
     ws = lzr.Workspace(nub, p, dev)
     ev = {}
 
@@ -280,32 +305,49 @@ def run_dedup_single(a):
             ev["d"][-1].record(stream)
         k = dedup_part()
         assert k == nu
-        lzr.gather_chunks(x, C, uniq, rank, ubuf)
+        lzr.gather_chunks(x, C, uniq, rank_, ubuf)
         launches[0] += lzr.last_launch_count()
         if record:
             ev.setdefault("e0", []).append(torch.cuda.Event(enable_timing=True))
             ev["e0"][-1].record(stream)
-        lzr.compress_encode(ubuf, p, ws)
+        lzr.compress_encode(ubuf[:nub], p, ws)
         launches[0] += lzr.last_launch_count()
         if record:
             ev.setdefault("e1", []).append(torch.cuda.Event(enable_timing=True))
             ev["e1"][-1].record(stream)
-        lzr.compress_compact(ubuf, p, ws)
+        lzr.compress_compact(ubuf[:nub], p, ws)
         launches[0] += lzr.last_launch_count()
+        if sharded:  # per-rank compressed totals -> global layout (8 B per rank)
+            dist.all_gather_into_tensor(totals_all, ws.total)
 
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
+    if sharded:
+        dist.barrier()
     launches[0] = 0
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(0) as clk:
+    with ClockSampler(local) as clk:
         torch.cuda.synchronize()
+        if sharded:
+            dist.barrier()
         t0.record(stream)
         for _ in range(a.steps):
             step(record=True)
         t1.record(stream)
         torch.cuda.synchronize()
-    ms_step = t0.elapsed_time(t1) / a.steps
+        if sharded:
+            dist.barrier()
+    ms = t0.elapsed_time(t1)
+    nub_all = nub
+    if sharded:
+        tt = torch.tensor([ms, float(nub)], dtype=torch.float64, device=dev)
+        mx = tt[:1].clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = tt[1:].clone()
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        ms, nub_all = float(mx.item()), int(sm.item())
+    ms_step = ms / a.steps
     enc_ms = [e0.elapsed_time(e1) for e0, e1 in zip(ev["e0"], ev["e1"])]
     dedup_ms = [d.elapsed_time(e0) for d, e0 in zip(ev["d"], ev["e0"])]
     assert int(index.overflow.item()) == 0
@@ -316,22 +358,25 @@ def run_dedup_single(a):
     enc_avg_s = statistics.mean(enc_ms) / 1e3
     hbm_peak, peak_src = peaks()
     achieved = enc_algo_bytes / enc_avg_s / 1e9
-    workload = (f"cfg5: {n >> 20} MiB logical mix dedup-2.0 stream ({nub >> 20} MiB unique), "
+    workload = (f"cfg5: {n_glob >> 20} MiB logical mix dedup-2.0 stream ({nub_all >> 20} MiB unique), "
                 f"dedup (SHA-1 + bin index + gather) then compress, C=W={C}, m=4, M=259")
     line = {
-        "metric": METRIC, "value": round(nub / (ms_step / 1e3) / 1e9, 4), "unit": UNIT,
-        "n_gpus": 1, "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 4),
+        "metric": METRIC, "value": round(nub_all / (ms_step / 1e3) / 1e9, 4), "unit": UNIT,
+        "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 4),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
-        "config": {"workload": workload, "global_bytes": n, "unique_bytes": nub,
-                   "dedup_ratio": round(N / nu, 4), "chunk_size": C, "window": C, "min_match": 4,
-                   "max_match": 259, "parallelism": "1 GPU",
+        "config": {"workload": workload, "global_bytes": n_glob, "unique_bytes": nub_all,
+                   "dedup_ratio": round(n_glob / max(1, nub_all), 4), "chunk_size": C, "window": C,
+                   "min_match": 4, "max_match": 259,
+                   "parallelism": (f"dp{world}: contiguous chunk shards; global index by NCCL "
+                                   "all-to-all to fingerprint owners; all-gather of totals")
+                   if sharded else "1 GPU",
                    "l2": "inputs larger than L2 (126 MB); no flush",
                    "compression_ratio": round(nub / max(1, total), 4),
                    "raw_chunk_fraction": round(float(raw.mean()), 4)},
-        "logical_value": round(n / (ms_step / 1e3) / 1e9, 4),
+        "logical_value": round(n_glob / (ms_step / 1e3) / 1e9, 4),
         "dedup": {"ms_per_step": round(statistics.mean(dedup_ms), 4),
-                  "logical_GBps": round(n / (statistics.mean(dedup_ms) / 1e3) / 1e9, 3),
+                  "logical_GBps": round(n_glob / (statistics.mean(dedup_ms) / 1e3) / 1e9, 3),
                   "what": "index reset + SHA-1 fingerprints + insert/lookup + unique scan + gather"},
         "roofline": {"bound": "hbm", "kernel": "lzr_encode_kernel", "achieved": round(achieved, 3),
                      "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 6),
@@ -342,7 +387,7 @@ def run_dedup_single(a):
         "clocks": clk.summary(),
         "gpu_launches": launches[0],
     }
-    if not a.no_cpu:
+    if grank == 0 and not a.no_cpu:
         import oracle
 
         smp = min(n, (a.cpu_sample_bytes // C) * C)
@@ -360,7 +405,10 @@ def run_dedup_single(a):
                                 "sample": f"first {smp >> 20} MiB of the logical stream: SHA-1, "
                                           f"index, compress of its {ub.size >> 20} MiB unique, {dt:.1f} s",
                                 "index_parity_vs_gpu": "bit-exact" if ok else "MISMATCH"}
-    print(json.dumps(line), flush=True)
+    if grank == 0:
+        print(json.dumps(line), flush=True)
+    if sharded:
+        dist.destroy_process_group()
 
 
 def main():
@@ -368,8 +416,8 @@ def main():
     if a.impl == "reference":
         run_reference(a)
         return
-    if a.config == 5 and "WORLD_SIZE" not in os.environ:
-        run_dedup_single(a)
+    if a.config == 5:
+        run_dedup(a)
         return
     import numpy as np
     import torch
@@ -391,9 +439,9 @@ def main():
     C = a.chunk_size
     p = lzr.Params(chunk_size=C)
     # workload (BASELINE.json configs); weak = fixed bytes per GPU, strong = fixed total
-    if a.config in (1, 4, 5):
+    if a.config in (1, 4):
         scaling = "strong"
-        n_glob = {1: 1 << 20, 4: 16 << 30, 5: 8 << 30}[a.config]
+        n_glob = {1: 1 << 20, 4: 16 << 30}[a.config]
         n_glob = (n_glob // C) * C
     else:
         scaling = "weak"
@@ -483,9 +531,6 @@ def main():
     achieved = enc_algo_bytes / enc_avg_s / 1e9
     if a.config == 2 and not a.bytes_per_rank:
         workload = f"cfg2: {n_rank >> 20} MiB {a.cls} per GPU, C=W={C}, m=4, M=259"
-    elif a.config == 5:
-        workload = (f"cfg5: {n_glob >> 20} MiB unique {a.cls} chunks of a {2 * n_glob >> 20} MiB "
-                    f"dedup-2.0 stream, sharded, C=W={C}, m=4, M=259")
     else:
         workload = (f"cfg{a.config}: {n_glob >> 20} MiB {a.cls} total ({scaling} scaling), "
                     f"C=W={C}, m=4, M=259")
@@ -569,8 +614,6 @@ def main():
                               + ("" if n_e2e == n_rank else f", first {n_e2e >> 20} MiB per GPU")}
         del scratch
 
-    if a.config == 5:
-        line["logical_value"] = round(2 * value, 4)  # logical (pre-dedup) bytes per second
     if rank == 0 and not a.no_cpu:
         smp = min(n_rank, (a.cpu_sample_bytes // C) * C) if a.config != 1 else n_rank
         ns = -(-smp // C)

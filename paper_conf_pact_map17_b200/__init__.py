@@ -18,7 +18,8 @@ __all__ = [
     "Params", "LzrError", "lib", "num_chunks", "compress_bound", "compress_workspace_bytes",
     "compress", "compress_encode", "compress_compact", "scan_sizes", "decompress",
     "compress_host", "validate_params", "status_str", "last_launch_count",
-    "fingerprint", "DedupIndex", "gather_chunks", "dedup_compress",
+    "fingerprint", "DedupIndex", "gather_chunks", "dedup_compress", "owner_counts", "route",
+    "unroute",
 ]
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
@@ -33,7 +34,8 @@ EXPORTED_SYMBOLS = [
     "lzr_scan_workspace_bytes", "lzr_scan_sizes", "lzr_decompress_chunks",
     "lzr_compress_host_scratch_bytes", "lzr_compress_host", "lzr_status_str",
     "lzr_last_launch_count", "lzr_fingerprint_chunks", "lzr_dedup_table_bytes", "lzr_dedup_index",
-    "lzr_gather_chunks",
+    "lzr_gather_chunks", "lzr_dedup_index_gidx", "lzr_dedup_owner_counts", "lzr_dedup_route",
+    "lzr_dedup_unroute",
 ]
 
 
@@ -104,6 +106,11 @@ def lib():
         L.lzr_dedup_index.argtypes = [vp, sz, u64, vp, ctypes.c_uint32, ctypes.c_uint32, vp, vp, vp,
                                       vp]
         L.lzr_gather_chunks.argtypes = [vp, sz, ctypes.c_uint32, vp, vp, vp, vp]
+        L.lzr_dedup_index_gidx.argtypes = [vp, sz, vp, vp, ctypes.c_uint32, ctypes.c_uint32, vp, vp,
+                                           vp, vp]
+        L.lzr_dedup_owner_counts.argtypes = [vp, sz, ctypes.c_uint32, vp, vp]
+        L.lzr_dedup_route.argtypes = [vp, sz, u64, ctypes.c_uint32, vp, vp, vp, vp, vp, vp]
+        L.lzr_dedup_unroute.argtypes = [vp, vp, sz, u64, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -328,6 +335,66 @@ class DedupIndex:
                                    _stream(stream, dev))
         _check(st, "lzr_dedup_index")
         return index[:N], unique[:N]
+
+    def index_gidx(self, fp, gidx, stream=None):
+        """Owner side of the multi-GPU index: record i's global index is gidx[i]."""
+        import torch
+
+        N = fp.shape[0]
+        dev = fp.device
+        index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+        unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+        st = lib().lzr_dedup_index_gidx(_ptr(fp), N, _ptr(gidx), _ptr(self.table), self.n_bins,
+                                        self.bin_slots, _ptr(index), _ptr(unique),
+                                        _ptr(self.overflow), _stream(stream, dev))
+        _check(st, "lzr_dedup_index_gidx")
+        return index[:N], unique[:N]
+
+
+def owner_counts(fp, n_owners: int, counts=None, stream=None):
+    """Per-owner fingerprint counts (int32[n_owners], zeroed here) for the
+    multi-GPU index (include/lzr.h lzr_dedup_owner_counts)."""
+    import torch
+
+    if counts is None:
+        counts = torch.zeros(n_owners, dtype=torch.int32, device=fp.device)
+    else:
+        counts.zero_()
+    st = lib().lzr_dedup_owner_counts(_ptr(fp), fp.shape[0], n_owners, _ptr(counts),
+                                      _stream(stream, fp.device))
+    _check(st, "lzr_dedup_owner_counts")
+    return counts
+
+
+def route(fp, first_chunk: int, n_owners: int, base, stream=None):
+    """Records (fingerprint, global index) grouped by owner in send order ->
+    (send_fp uint8[N,20], send_gidx int64[N], slot int32[N])."""
+    import torch
+
+    N = fp.shape[0]
+    dev = fp.device
+    cursor = torch.zeros(n_owners, dtype=torch.int32, device=dev)
+    send_fp = torch.empty((max(1, N), 20), dtype=torch.uint8, device=dev)
+    send_gidx = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+    slot = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+    st = lib().lzr_dedup_route(_ptr(fp), N, first_chunk, n_owners, _ptr(base), _ptr(cursor),
+                               _ptr(send_fp), _ptr(send_gidx), _ptr(slot), _stream(stream, dev))
+    _check(st, "lzr_dedup_route")
+    return send_fp[:N], send_gidx[:N], slot[:N]
+
+
+def unroute(back, slot, first_chunk: int, stream=None):
+    """Owners' index numbers (send order) -> (index int64[N], unique int32[N]) in chunk order."""
+    import torch
+
+    N = slot.shape[0]
+    dev = slot.device
+    index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+    unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+    st = lib().lzr_dedup_unroute(_ptr(back), _ptr(slot), N, first_chunk, _ptr(index), _ptr(unique),
+                                 _stream(stream, dev))
+    _check(st, "lzr_dedup_unroute")
+    return index[:N], unique[:N]
 
 
 def gather_chunks(t, chunk_size: int, unique, rank, out, stream=None):

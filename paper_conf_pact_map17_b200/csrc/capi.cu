@@ -279,8 +279,64 @@ int lzr_dedup_index(const uint8_t* d_fp, size_t n_chunks, uint64_t first_chunk, 
   if (!aligned(d_table, 256) || !aligned(d_index, 8) || !aligned(d_unique, 4) ||
       !aligned(d_overflow, 4))
     return LZR_ERR_INVALID_ARG;
-  if (launch_index(d_fp, n_chunks, first_chunk, d_table, n_bins, bin_slots, d_index, d_unique,
-                   d_overflow, (cudaStream_t)stream, &t_launches) != cudaSuccess)
+  if (launch_index(d_fp, n_chunks, first_chunk, nullptr, d_table, n_bins, bin_slots, d_index,
+                   d_unique, d_overflow, (cudaStream_t)stream, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_dedup_index_gidx(const uint8_t* d_fp, size_t n, const uint64_t* d_gidx, void* d_table,
+                         uint32_t n_bins, uint32_t bin_slots, uint64_t* d_index, uint32_t* d_unique,
+                         uint32_t* d_overflow, lzr_stream_t stream) {
+  t_launches = 0;
+  if (n == 0) return LZR_OK;
+  if (!d_fp || !d_gidx || !d_table || !d_index || !d_unique || !d_overflow || n_bins == 0 ||
+      bin_slots == 0)
+    return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_table, 256) || !aligned(d_gidx, 8) || !aligned(d_index, 8) || !aligned(d_unique, 4) ||
+      !aligned(d_overflow, 4))
+    return LZR_ERR_INVALID_ARG;
+  if (launch_index(d_fp, n, 0, d_gidx, d_table, n_bins, bin_slots, d_index, d_unique, d_overflow,
+                   (cudaStream_t)stream, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_dedup_owner_counts(const uint8_t* d_fp, size_t n, uint32_t n_owners, uint32_t* d_counts,
+                           lzr_stream_t stream) {
+  t_launches = 0;
+  if (n == 0) return LZR_OK;
+  if (!d_fp || !d_counts || n_owners == 0 || !aligned(d_counts, 4)) return LZR_ERR_INVALID_ARG;
+  if (launch_owner_counts(d_fp, n, n_owners, d_counts, (cudaStream_t)stream, &t_launches) !=
+      cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_dedup_route(const uint8_t* d_fp, size_t n, uint64_t first_chunk, uint32_t n_owners,
+                    const uint64_t* d_base, uint32_t* d_cursor, uint8_t* d_send_fp,
+                    uint64_t* d_send_gidx, uint32_t* d_slot, lzr_stream_t stream) {
+  t_launches = 0;
+  if (n == 0) return LZR_OK;
+  if (!d_fp || !d_base || !d_cursor || !d_send_fp || !d_send_gidx || !d_slot || n_owners == 0)
+    return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_base, 8) || !aligned(d_cursor, 4) || !aligned(d_send_gidx, 8) || !aligned(d_slot, 4))
+    return LZR_ERR_INVALID_ARG;
+  if (launch_route(d_fp, n, first_chunk, n_owners, d_base, d_cursor, d_send_fp, d_send_gidx, d_slot,
+                   (cudaStream_t)stream, &t_launches) != cudaSuccess)
+    return LZR_ERR_CUDA;
+  return LZR_OK;
+}
+
+int lzr_dedup_unroute(const uint64_t* d_back, const uint32_t* d_slot, size_t n, uint64_t first_chunk,
+                      uint64_t* d_index, uint32_t* d_unique, lzr_stream_t stream) {
+  t_launches = 0;
+  if (n == 0) return LZR_OK;
+  if (!d_back || !d_slot || !d_index || !d_unique) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_back, 8) || !aligned(d_slot, 4) || !aligned(d_index, 8) || !aligned(d_unique, 4))
+    return LZR_ERR_INVALID_ARG;
+  if (launch_unroute(d_back, d_slot, n, first_chunk, d_index, d_unique, (cudaStream_t)stream,
+                     &t_launches) != cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;
 }

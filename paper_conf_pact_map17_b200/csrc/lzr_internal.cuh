@@ -174,9 +174,16 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
 cudaError_t launch_sha1(const uint8_t* in, size_t n, uint32_t C, uint8_t* fp, cudaStream_t s,
                         int* launches);
 size_t dedup_entry_bytes();
-cudaError_t launch_index(const uint8_t* fps, size_t N, uint64_t first, void* table, uint32_t n_bins,
-                         uint32_t bin_slots, uint64_t* index, uint32_t* unique, uint32_t* overflow,
-                         cudaStream_t s, int* launches);
+cudaError_t launch_index(const uint8_t* fps, size_t N, uint64_t first, const uint64_t* gidx,
+                         void* table, uint32_t n_bins, uint32_t bin_slots, uint64_t* index,
+                         uint32_t* unique, uint32_t* overflow, cudaStream_t s, int* launches);
+cudaError_t launch_owner_counts(const uint8_t* fps, size_t N, uint32_t n_owners, uint32_t* counts,
+                                cudaStream_t s, int* launches);
+cudaError_t launch_route(const uint8_t* fps, size_t N, uint64_t first, uint32_t n_owners,
+                         const uint64_t* base, uint32_t* cursor, uint8_t* send_fp, uint64_t* send_gidx,
+                         uint32_t* slot, cudaStream_t s, int* launches);
+cudaError_t launch_unroute(const uint64_t* back, const uint32_t* slot, size_t N, uint64_t first,
+                           uint64_t* index, uint32_t* unique, cudaStream_t s, int* launches);
 cudaError_t launch_gather(const uint8_t* in, size_t n, uint32_t C, const uint32_t* unique,
                           const uint64_t* rank, uint8_t* out, int sm_count, cudaStream_t s,
                           int* launches);

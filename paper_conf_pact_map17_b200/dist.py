@@ -23,7 +23,8 @@ from dataclasses import dataclass
 import torch
 import torch.distributed as dist
 
-from . import Params, Workspace, compress, num_chunks, scan_sizes
+from . import (DedupIndex, Params, Workspace, compress, fingerprint, num_chunks, owner_counts, route,
+               scan_sizes, unroute)
 
 
 def shard_range(n_chunks: int, world: int, rank: int) -> tuple[int, int]:
@@ -126,3 +127,82 @@ class ShardedCompressor:
 def compress_sharded(x_local, p: Params, n_bytes_global: int, group=None):
     """One-shot convenience wrapper (allocates buffers every call)."""
     return ShardedCompressor(n_bytes_global, p, group, x_local.device)(x_local)
+
+
+# ---- multi-GPU dedup (DESIGN.md §11; SURVEY.md §8(f) N2 across ranks) ------------
+class CudaDedupOps:
+    """The product path of ShardedDedup: liblzr kernels + torch.distributed."""
+
+    def __init__(self, index: DedupIndex):
+        self.index = index
+
+    def fingerprint(self, x, C):
+        return fingerprint(x, C)
+
+    def owner_counts(self, fp, R):
+        return owner_counts(fp, R)
+
+    def route(self, fp, first, R, base):
+        return route(fp, first, R, base)
+
+    def index_gidx(self, fp, gidx):
+        return self.index.index_gidx(fp, gidx)[0]
+
+    def unroute(self, back, slot, first):
+        return unroute(back, slot, first)
+
+    def all_to_all(self, out, inp, out_splits, in_splits, group):
+        dist.all_to_all_single(out, inp, output_split_sizes=out_splits,
+                               input_split_sizes=in_splits, group=group)
+
+
+class ShardedDedup:
+    """Global dedup of a stream sharded over R ranks (contiguous chunk ranges).
+
+    The index is partitioned over the ranks by fingerprint (owner = third
+    fingerprint word scaled to R; §3.1(1) bins, spread over GPUs).  One
+    call: fingerprint the local chunks; count and route (fingerprint, global
+    chunk index) records to their owners (all-to-all of the counts, then of the
+    records: the real exchange step of dedup); each owner inserts and looks up
+    everything it received in its own DedupIndex (insert-or-min, so the index
+    number = the first occurrence in the global stream, wherever it lives);
+    the index numbers go back by the reverse all-to-all and are put back in
+    chunk order.  Result per local chunk: (index number, unique flag) equal to
+    single-process indexing of the whole stream (R18).
+    """
+
+    def __init__(self, n_local_max: int, group=None, device=None, ops=None, bin_slots: int = 64,
+                 skew: float = 1.5):
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        if ops is None:
+            # an owner receives ~n_local chunks on average; skew covers imbalance
+            cap = int(skew * max(1, n_local_max)) + 1024
+            ops = CudaDedupOps(DedupIndex.for_chunks(cap, device, bin_slots))
+        self.ops = ops
+
+    def __call__(self, x_local, chunk_size: int, first_chunk: int):
+        R = self.world
+        fp = self.ops.fingerprint(x_local, chunk_size)
+        N = fp.shape[0]
+        dev = fp.device
+        counts = self.ops.owner_counts(fp, R).to(torch.int64)
+        recv_counts = torch.empty_like(counts)
+        self.ops.all_to_all(recv_counts, counts, None, None, self.group)
+        in_splits = counts.cpu().tolist()
+        out_splits = recv_counts.cpu().tolist()
+        base = torch.zeros(R, dtype=torch.int64, device=dev)
+        if R > 1:
+            base[1:] = torch.cumsum(counts, 0)[:-1]
+        send_fp, send_gidx, slot = self.ops.route(fp, first_chunk, R, base)
+        n_recv = int(sum(out_splits))
+        recv_fp = torch.empty((n_recv, 20), dtype=torch.uint8, device=dev)
+        recv_gidx = torch.empty(n_recv, dtype=torch.int64, device=dev)
+        self.ops.all_to_all(recv_fp, send_fp, out_splits, in_splits, self.group)
+        self.ops.all_to_all(recv_gidx, send_gidx, out_splits, in_splits, self.group)
+        recv_index = self.ops.index_gidx(recv_fp, recv_gidx) if n_recv else recv_gidx
+        back = torch.empty(N, dtype=torch.int64, device=dev)
+        self.ops.all_to_all(back, recv_index, in_splits, out_splits, self.group)
+        index, unique = self.ops.unroute(back, slot, first_chunk)
+        return fp, index, unique

@@ -115,3 +115,106 @@ def test_sharded_offsets_match_single_process(ref, world, nchunks, tail):
         got = np.concatenate([sizes_all.view(np.uint32)[r * mx: r * mx + (shard_range(N, world, r)[1] - shard_range(N, world, r)[0])]
                               for r in range(world)])
         assert np.array_equal(got, r_sizes)
+
+
+# ---- multi-rank dedup (ShardedDedup): host-side routing over gloo -----------------
+class OracleDedupOps:
+    """CPU stand-in for CudaDedupOps (test only): oracle fingerprints, a numpy
+    owner partition and router, and a dict index with insert-or-min semantics."""
+
+    def __init__(self):
+        import oracle
+
+        self.ref = oracle
+        self.table = {}
+
+    def fingerprint(self, x, C):
+        return torch.from_numpy(self.ref.fingerprints(x.numpy(), C, n_threads=1).copy())
+
+    @staticmethod
+    def _owner(fp, R):
+        w2 = (fp[:, 8].astype(np.uint64) << 24) | (fp[:, 9].astype(np.uint64) << 16) | \
+             (fp[:, 10].astype(np.uint64) << 8) | fp[:, 11].astype(np.uint64)
+        return ((w2 * np.uint64(R)) >> np.uint64(32)).astype(np.int64)
+
+    def owner_counts(self, fp, R):
+        return torch.from_numpy(np.bincount(self._owner(fp.numpy(), R), minlength=R).astype(np.int32))
+
+    def route(self, fp, first, R, base):
+        f = fp.numpy()
+        own = self._owner(f, R)
+        order = np.argsort(own, kind="stable")
+        slot = np.empty(len(f), np.int32)
+        slot[order] = np.arange(len(f), dtype=np.int32)
+        gidx = first + np.arange(len(f), dtype=np.int64)
+        return torch.from_numpy(f[order].copy()), torch.from_numpy(gidx[order].copy()), torch.from_numpy(slot)
+
+    def index_gidx(self, fp, gidx):
+        f, g = fp.numpy(), gidx.numpy()
+        for k in range(len(f)):  # insert-or-min over the whole batch first
+            key = f[k].tobytes()
+            self.table[key] = min(self.table.get(key, int(g[k])), int(g[k]))
+        return torch.tensor([self.table[f[k].tobytes()] for k in range(len(f))], dtype=torch.int64)
+
+    def unroute(self, back, slot, first):
+        idx = back.numpy()[slot.numpy()]
+        uniq = (idx == first + np.arange(len(idx))).astype(np.int32)
+        return torch.from_numpy(idx.copy()), torch.from_numpy(uniq)
+
+    def all_to_all(self, out, inp, out_splits, in_splits, group):
+        dist.all_to_all_single(out, inp, output_split_sizes=out_splits, input_split_sizes=in_splits,
+                               group=group)
+
+
+def _dedup_worker(rank, world, port, n_chunks, C, rounds, q):
+    """The stream is indexed in `rounds` global batches (stream order); each
+    batch is sharded over the ranks by contiguous chunk ranges."""
+    import synth
+    from paper_conf_pact_map17_b200.dist import ShardedDedup
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        x = synth.fill_host(n_chunks * C, C, "mix_dedup")
+        per = -(-n_chunks // rounds)
+        sd = ShardedDedup(per, ops=OracleDedupOps())
+        outs = []
+        for b in range(rounds):
+            g0, g1 = b * per, min(n_chunks, (b + 1) * per)
+            lo, hi = shard_range(g1 - g0, world, rank)
+            lo, hi = g0 + lo, g0 + hi
+            _, idx, un = sd(torch.from_numpy(np.ascontiguousarray(x[lo * C:hi * C])), C, lo)
+            outs.append((lo, idx.numpy().copy(), un.numpy().copy()))
+        q.put((rank, outs))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,rounds", [(2, 1), (3, 1), (2, 3), (4, 2)])
+def test_sharded_dedup_matches_single_process(ref, world, rounds):
+    import synth
+
+    C, n_chunks = 256, 300
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_dedup_worker, args=(r, world, port, n_chunks, C, rounds, q))
+             for r in range(world)]
+    for pr in procs:
+        pr.start()
+    results = [q.get(timeout=180) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    x = synth.fill_host(n_chunks * C, C, "mix_dedup")
+    r_idx, r_hit, _ = ref.dedup_index(ref.fingerprints(x, C), 0)
+    assert r_hit.sum() > 0.3 * n_chunks  # the stream does carry cross-shard duplicates
+    got_idx = np.zeros(n_chunks, np.int64) - 1
+    got_un = np.zeros(n_chunks, np.int32) - 1
+    for rank, outs in results:
+        for b0, idx, un in outs:
+            got_idx[b0:b0 + len(idx)] = idx
+            got_un[b0:b0 + len(un)] = un
+    assert np.array_equal(got_idx.astype(np.uint64), r_idx)
+    assert np.array_equal(got_un.astype(bool), ~r_hit.astype(bool))
