@@ -44,7 +44,7 @@ constexpr uint16_t kPos = 0x7FFF;
 
 // ctrl word indices (per group): chunk, U, nruns, then prog[K], sync[K] during
 // the walk, reused as T[K], M[K] (token / match totals) after the chain phase
-constexpr int kCtrlChunk = 0, kCtrlU = 1, kCtrlRuns = 2, kCtrlProg = 4;
+constexpr int kCtrlChunk = 0, kCtrlU = 1, kCtrlRuns = 2, kCtrlIdx = 3, kCtrlProg = 4;
 
 // Bucket of a key.  With >= 1024 buckets, keys that are one repeated byte get
 // private buckets 0..255 (their buckets can hold thousands of positions, e.g.
@@ -601,6 +601,12 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
       continue;
     }
     const uint32_t nruns = S.ctrl[kCtrlRuns];
+    // Positions whose key is one repeated byte are searched by the run-aware
+    // search only (best_match_runs) when every run fits the run list and every
+    // position's whole prefix is in the window; then they need no index entry:
+    // their private buckets (< 256) are left empty and their candidate bits come
+    // from the run structure (below).  Zero-run chunks skip most of the scatter.
+    const bool skipr = hb >= 10 && nruns <= a.L.max_runs && a.W + 1 >= n;
 
     // ---- warp 0: exclusive scan of the B bucket totals (2 buckets per lane and
     //      round); split j's cursor of bucket h = start of h + counts of h in
@@ -611,9 +617,10 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
       uint32_t carry = 0;
       for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
         const bool act = w0 + lane < B / 2;
+        const bool priv = skipr && w0 + lane < 128;  // buckets 2w, 2w+1 < 256: left empty
         uint32_t c0 = 0, c1 = 0;  // totals of buckets 2w, 2w+1
         for (uint32_t j = 0; j < NS; ++j) {
-          const uint32_t wv = act ? hist[j * (B / 2) + w0 + lane] : 0;
+          const uint32_t wv = act && !priv ? hist[j * (B / 2) + w0 + lane] : 0;
           c0 += wv & 0xFFFFu;
           c1 += wv >> 16;
         }
@@ -627,7 +634,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
         uint32_t e0 = incl - sum + carry, e1 = e0 + c0;  // running cursors
         if (act) {
           for (uint32_t j = 0; j < NS; ++j) {
-            const uint32_t wv = hist[j * (B / 2) + w0 + lane];
+            const uint32_t wv = priv ? 0u : hist[j * (B / 2) + w0 + lane];
             hist[j * (B / 2) + w0 + lane] = (e0 & 0xFFFFu) | (e1 << 16);
             e0 += wv & 0xFFFFu;
             e1 += wv >> 16;
@@ -635,6 +642,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
         }
         carry += __shfl_sync(kFull, incl, 31);
       }
+      if (lane == 0) S.ctrl[kCtrlIdx] = carry;  // index entries (P, or fewer when skipr)
     }
     if (K == 1 || k != 0) {
       for (uint32_t i = kk * 32 + lane; i < nw; i += KK * 32) S.cand[i] = 0;
@@ -666,15 +674,15 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
         for (int u = 0; u < 4; ++u) {
           const uint32_t p = p0 + 32 * u + lane;
           h[u] = p < pe ? khash(ld32u(S.data, p) & a.kmask, hb, a.kmask) : 0xFFFFFFFFu;
+          if (skipr && h[u] < 256u) h[u] = 0xFFFFFFFFu;  // not indexed
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          const uint32_t p = p0 + 32 * u + lane;
-          const bool act = p < pe;
+          const bool act = h[u] != 0xFFFFFFFFu;
           const uint32_t basev = act ? cur[h[u]] : 0;
-          if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)p;
+          if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)(p0 + 32 * u + lane);
           __syncwarp();
           if (act && lane == 31u - __clz(peers[u])) cur[h[u]] = (uint16_t)(basev + __popc(peers[u]));
           __syncwarp();
@@ -702,7 +710,8 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
 
     // ---- slot of each position and the candidate bitmap: the nearest same-key
     //      earlier position is the nearest same-key entry below in the bucket
-    for (uint32_t sl = tid; sl < P; sl += nthr) {
+    const uint32_t nidx = S.ctrl[kCtrlIdx];
+    for (uint32_t sl = tid; sl < nidx; sl += nthr) {
       const uint32_t e = S.sorted[sl];
       const uint32_t q = e & kPos;
       S.slot[q] = (uint16_t)sl;
@@ -719,6 +728,29 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
           if (e2 & kFirst) break;
         }
         if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
+      }
+    }
+    if (skipr && nruns) {
+      // not-indexed positions (key = k copies of one byte): inside a run (the
+      // byte before is the same) the key also occurs at d = 1; a run start has a
+      // candidate iff an earlier run of the same byte (length >= k) exists
+      for (uint32_t w = tid; w < (P + 31) >> 5; w += nthr) {
+        const uint32_t c0 = S.cb[w], c1 = S.cb[w + 1];
+        uint32_t z = c0;  // cb bit p (byte p differs from p-1) ...
+        for (uint32_t j = 1; j < a.kbytes; ++j) z |= __funnelshift_r(c0, c1, j);  // ... or p+1..p+k-1
+        const uint32_t mrun = ~z & valid_mask(P, w);
+        if (mrun) atomicOr(&S.cand[w], mrun);
+      }
+      if (k == 0) {
+        for (uint32_t j = lane; j < nruns; j += 32) {
+          const uint32_t st = S.runs[j] & 0xFFFFu, b = S.data[st];
+          bool has = false;
+          for (uint32_t i = 0; i < nruns && !has; ++i) {
+            const uint32_t t = S.runs[i] & 0xFFFFu;
+            has = t < st && S.data[t] == b;
+          }
+          if (has && st < P) atomicOr(&S.cand[st >> 5], 1u << (st & 31u));
+        }
       }
     }
     GSYNC(6);

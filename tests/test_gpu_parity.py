@@ -316,3 +316,22 @@ def test_gpu_decoder_fuzz_vs_oracle(lzr, ref, C, m, cls):
         if r_bad == 0:
             n_valid += 1
             assert np.array_equal(y.cpu().numpy(), r_y), trial
+
+
+@pytest.mark.parametrize("C,W,m", [(4096, 4096, 3), (4096, 4096, 5), (8192, 8192, 4), (32768, 32768, 4),
+                                   (4096, 4095, 4), (4096, 4094, 4), (8192, 8192, 3)])
+def test_runs_structures_param_grid(lzr, ref, C, W, m):
+    """Run-heavy chunks across m, C and W around the 'every prefix in the window'
+    boundary: the index leaves repeated-byte keys out (run-aware search only) iff
+    the runs fit the run list and W + 1 >= n; both sides of that switch must give
+    the oracle's bytes."""
+    rng = np.random.default_rng(C + W + m)
+    parts = []
+    for k in range(3000):
+        parts.append(np.full(int(rng.integers(1, 70)), int(rng.integers(0, 4)), np.uint8))
+        if k % 5 == 0:
+            parts.append(rng.integers(0, 256, int(rng.integers(1, 12)), dtype=np.uint8))
+    x = np.concatenate(parts)[: C * 4 + 333]
+    _check_full(lzr, ref, x, lzr.Params(chunk_size=C, window=W, min_match=m))
+    z = synth.fill_host(C * 6, C, "zeroruns", seed=m)
+    _check_full(lzr, ref, z, lzr.Params(chunk_size=C, window=W, min_match=m))
