@@ -1,5 +1,6 @@
 #!/bin/bash
-# compute-sanitizer over the compress + decompress path on small inputs (run under gpurun)
+# compute-sanitizer over the compress + decompress path (4 KiB and 8 KiB chunks)
+# and the dedup path on small inputs (run under gpurun)
 out=gpurun_out/sanitize
 mkdir -p $out
 for tool in memcheck racecheck synccheck initcheck; do
@@ -8,4 +9,9 @@ for tool in memcheck racecheck synccheck initcheck; do
       python tools/prof_encode.py --cls $cls --mib 2 --iters 1 --decode > $out/${tool}_${cls}.log 2>&1
     echo "$tool $cls rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_${cls}.log | tail -1)"
   done
+  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 \
+    python tools/prof_encode.py --cls mix --mib 2 --iters 1 --decode --chunk-size 8192 > $out/${tool}_mix8k.log 2>&1
+  echo "$tool mix C=8192 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_mix8k.log | tail -1)"
+  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/prof_dedup.py > $out/${tool}_dedup.log 2>&1
+  echo "$tool dedup rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_dedup.log | tail -1)"
 done
