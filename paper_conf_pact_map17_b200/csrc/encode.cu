@@ -406,8 +406,13 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
 __device__ __forceinline__ uint32_t walk_bound(uint32_t n, uint32_t k, uint32_t K) {
   if (k == 0) return 0;
   if (k >= K) return n;
-  // density 1 + 0.5 x  =>  bound = (sqrt(1 + 1.25 k/K) - 1) / 0.5
-  const float f = 2.0f * (sqrtf(1.0f + 1.25f * (float)k / (float)K) - 1.0f);
+#ifndef LZR_WALK_C
+#define LZR_WALK_C 0.5f
+#endif
+  // work density 1 + c x over the chunk (later positions have more candidates)
+  // => bound x solves x + c x^2 / 2 = (k/K)(1 + c/2)
+  constexpr float c = LZR_WALK_C;
+  const float f = (sqrtf(1.0f + 2.0f * c * (1.0f + 0.5f * c) * (float)k / (float)K) - 1.0f) / c;
   const uint32_t b = (uint32_t)(f * (float)n);
   return b < n ? b : n;
 }
