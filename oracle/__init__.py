@@ -35,6 +35,7 @@ class _Params(ctypes.Structure):
         ("min_match", ctypes.c_uint32),
         ("max_match", ctypes.c_uint32),
         ("tie_break", ctypes.c_uint32),
+        ("parse", ctypes.c_uint32),
     ]
 
 
@@ -45,11 +46,12 @@ class Params:
     min_match: int = 4
     max_match: int | None = None  # None -> min_match + 255
     tie_break: int = 0
+    parse: int = 0  # 0 = greedy (R8), 1 = one-step lazy (R21)
 
     def c(self) -> _Params:
         w = self.chunk_size if self.window is None else self.window
         mm = self.min_match + 255 if self.max_match is None else self.max_match
-        return _Params(self.chunk_size, w, self.min_match, mm, self.tie_break)
+        return _Params(self.chunk_size, w, self.min_match, mm, self.tie_break, self.parse)
 
 
 _lib = None

@@ -18,7 +18,8 @@
 
 /* R-params (R1, R3, R4, R7): C multiple of 16 in [16, 65536];
  * 1 <= W <= C; 3 <= m <= 255; m <= M <= m + 255 (8-bit length field);
- * tie_break must be 0 ("longest, then nearest"). */
+ * tie_break must be 0 ("longest, then nearest"); parse 0 (greedy, R8) or 1
+ * (one-step lazy, R21). */
 int lzr_ref_validate(const lzr_ref_params* p) {
   if (!p) return LZR_REF_ERR_INVALID_ARG;
   if (p->chunk_size < 16 || p->chunk_size > 65536 || (p->chunk_size % 16) != 0)
@@ -28,6 +29,7 @@ int lzr_ref_validate(const lzr_ref_params* p) {
   if (p->max_match < p->min_match || p->max_match > p->min_match + 255)
     return LZR_REF_ERR_INVALID_ARG;
   if (p->tie_break != 0) return LZR_REF_ERR_UNSUPPORTED;
+  if (p->parse > 1) return LZR_REF_ERR_UNSUPPORTED;
   return LZR_REF_OK;
 }
 
@@ -67,14 +69,24 @@ void lzr_ref_best_match(const uint8_t* x, size_t n, size_t p, const lzr_ref_para
 
 /* Greedy parse (R8; §3.2(2) post-processing, whose rule the paper does
  * not give): p = 0; while p < n: take the best match if its length >= m,
- * else a literal. */
+ * else a literal.
+ * One-step lazy parse (R21, parse = 1; SURVEY.md §8(f) N4 "lazy matching"):
+ * the same, except that a match at p is deferred -- x[p] is emitted as a
+ * literal and the walk moves to p + 1 -- when the best match at p + 1 is
+ * strictly longer than the one at p.  The decision at p depends on p alone. */
 size_t lzr_ref_parse_chunk(const uint8_t* x, size_t n, const lzr_ref_params* prm,
                            uint32_t* lens, uint32_t* dists) {
   size_t p = 0, t = 0;
   while (p < n) {
     uint32_t l, d;
     lzr_ref_best_match(x, n, p, prm, &l, &d);
-    if (l >= prm->min_match) {
+    int take = l >= prm->min_match;
+    if (take && prm->parse == 1 && p + 1 < n) {
+      uint32_t l1, d1;
+      lzr_ref_best_match(x, n, p + 1, prm, &l1, &d1);
+      if (l1 > l) take = 0; /* a longer match starts at p + 1: literal now */
+    }
+    if (take) {
       lens[t] = l;
       dists[t] = d;
       p += l;

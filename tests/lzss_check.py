@@ -6,6 +6,9 @@
 * ``brute_tokens``: the greedy longest-then-nearest parse recomputed by brute
   force in a different formulation (full table of capped common-prefix lengths
   for every admissible distance, then argmax) -- only for tiny inputs.
+* ``brute_tokens_lazy``: the one-step lazy parse (R21) from a
+  precomputed table of best (length, distance) at every position, then a walk
+  over the table -- a different formulation from the oracle's on-the-fly one.
 * ``check_tokens``: properties every correct token stream satisfies.
 """
 from __future__ import annotations
@@ -68,6 +71,34 @@ def brute_tokens(x: bytes, W: int, m: int, M: int):
             d = min(d for d, l in tab if l == best)
             toks.append((best, d))
             p += best
+        else:
+            toks.append((1, 0))
+            p += 1
+    return toks
+
+
+def best_table(x: bytes, W: int, M: int):
+    """[(l*, d*)] at every position: longest capped match, smallest d among equals."""
+    out = []
+    for p in range(len(x)):
+        tab = capped_lcp_table(x, p, W, M)
+        best = max((l for _, l in tab), default=0)
+        d = min((d for d, l in tab if l == best), default=0) if best else 0
+        out.append((best, d))
+    return out
+
+
+def brute_tokens_lazy(x: bytes, W: int, m: int, M: int):
+    n = len(x)
+    bt = best_table(x, W, M)
+    p = 0
+    toks = []
+    while p < n:
+        l, d = bt[p]
+        deferred = p + 1 < n and bt[p + 1][0] > l
+        if l >= m and not deferred:
+            toks.append((l, d))
+            p += l
         else:
             toks.append((1, 0))
             p += 1

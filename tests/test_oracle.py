@@ -23,12 +23,16 @@ import pytest
 
 from tests import lzss_check as lc
 
-GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "appendix_a.jsonl")
+GOLDEN = [os.path.join(os.path.dirname(__file__), "golden", f)
+          for f in ("appendix_a.jsonl", "lazy_examples.jsonl")]
 
 
 def _golden():
-    with open(GOLDEN) as f:
-        return [json.loads(l) for l in f if l.strip()]
+    out = []
+    for path in GOLDEN:
+        with open(path) as f:
+            out += [json.loads(l) for l in f if l.strip()]
+    return out
 
 
 def _params(ref, d):
@@ -167,6 +171,67 @@ def test_bruteforce_random_strings(ref):
         assert st == 0 and y == x
 
 
+# ---- one-step lazy parse (R21) -----------------
+
+def test_lazy_bruteforce_all_binary_strings(ref):
+    checked = differ = 0
+    for n in range(1, 11):
+        for tup in itertools.product(b"ab", repeat=n):
+            x = bytes(tup)
+            for W, m, M in _grid(n):
+                if W > 16:
+                    continue
+                p = ref.Params(chunk_size=16, window=W, min_match=m, max_match=M, parse=1)
+                toks = ref.parse_chunk(x, p)
+                assert toks == lc.brute_tokens_lazy(x, W, m, M), (x, W, m, M)
+                differ += toks != lc.brute_tokens(x, W, m, M)
+                checked += 1
+    assert checked > 10000 and differ > 100  # the two parses really differ
+
+
+def test_lazy_bruteforce_random_strings(ref):
+    rng = random.Random(0x1A2F)
+    for it in range(2000):
+        n = rng.randint(1, 64)
+        alpha = rng.choice([2, 4, 256])
+        x = bytes(rng.randrange(alpha) for _ in range(n))
+        W = max(1, rng.choice([1, 2, 3, 5, 8, n]))
+        m = rng.choice([3, 4, 5])
+        M = m + rng.choice([0, 1, 3, 255])
+        p = ref.Params(chunk_size=64, window=W, min_match=m, max_match=M, parse=1)
+        toks = ref.parse_chunk(x, p)
+        assert toks == lc.brute_tokens_lazy(x, W, m, M), (x, W, m, M)
+        lc.check_tokens(x, toks, W, m, M)
+        s = ref.compress_chunk(x, p)
+        if len(s) < n:
+            assert lc.parse_stream(s, n, m) == toks
+        st, y = ref.decompress_chunk(s, n, p)
+        assert st == 0 and y == x
+
+
+def test_lazy_equals_greedy_on_constant_and_periodic(ref):
+    # the best length never grows from p to p+1 on constant / periodic data
+    # (it is min(M, n-p) once the first period is history), so nothing is
+    # deferred: the closed forms of the greedy parse hold unchanged
+    for n in (4096, 8192):
+        p = ref.Params(chunk_size=n, parse=1)
+        assert len(ref.compress_chunk(bytes(n), p)) == _const_closed_form(n, 4, 259)
+    for q in [1, 2, 3, 5, 7, 31, 255]:
+        x = bytes((i % q) + 1 for i in range(4096))
+        assert ref.parse_chunk(x, ref.Params(parse=1)) == ref.parse_chunk(x, ref.Params())
+
+
+def test_lazy_stream_roundtrip(ref):
+    import synth
+    x = synth.fill_host(64 * 4096, 4096, "mix", seed=5)
+    p = ref.Params(parse=1)
+    out, sizes, offsets, total = ref.compress(x, p)
+    st, bad, y = ref.decompress(out, sizes, offsets, x.size, p)
+    assert st == 0 and bad == 0 and np.array_equal(y, x)
+    _, g_sizes, _, _ = ref.compress(x, ref.Params())
+    assert not np.array_equal(sizes, g_sizes)  # lazy changes some chunks
+
+
 def test_param_validation(ref):
     P = ref.Params
     assert ref.validate(P()) == 0
@@ -179,6 +244,8 @@ def test_param_validation(ref):
     assert ref.validate(P(min_match=4, max_match=3)) == ref.ERR_INVALID_ARG
     assert ref.validate(P(min_match=4, max_match=260)) == ref.ERR_INVALID_ARG
     assert ref.validate(P(tie_break=1)) == ref.ERR_UNSUPPORTED
+    assert ref.validate(P(parse=1)) == ref.OK
+    assert ref.validate(P(parse=2)) == ref.ERR_UNSUPPORTED
 
 
 def _mixed_stream(n, seed):
