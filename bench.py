@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-decode", action="store_true")
+    ap.add_argument("--parse", default="greedy", choices=["greedy", "lazy"],
+                    help="parse rule (DESIGN.md R8 greedy, R21 one-step lazy; SURVEY.md §8(f) N4)")
     return ap.parse_args()
 
 
@@ -175,7 +177,8 @@ def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
     xs = x_host[: nchunks * C]
     cores = len(os.sched_getaffinity(0))
     t0 = time.perf_counter()
-    r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, oracle.Params(chunk_size=C), n_threads=cores)
+    r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, oracle.Params(chunk_size=C, parse=p_gpu.parse),
+                                                   n_threads=cores)
     dt = time.perf_counter() - t0
     ok = bool(np.array_equal(r_sizes, g_sizes[:nchunks]) and np.array_equal(r_offs, g_offs[:nchunks])
               and np.array_equal(r_out, g_out[: int(r_tot)]))
@@ -183,6 +186,9 @@ def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
             "sample": f"first {nchunks} chunks ({xs.size / 2**20:.0f} MiB) of the timed stream, "
                       f"thread-per-chunk, {dt:.1f} s",
             "parity_vs_gpu": "bit-exact" if ok else "MISMATCH"}
+
+
+PARSES = {"greedy": 0, "lazy": 1}  # lzr_params.parse (include/lzr.h)
 
 
 def run_reference(a):
@@ -198,7 +204,7 @@ def run_reference(a):
     C = a.chunk_size
     cores = len(os.sched_getaffinity(0))
     n = (a.ref_sample_bytes // C) * C
-    p = oracle.Params(chunk_size=C)
+    p = oracle.Params(chunk_size=C, parse=PARSES[a.parse])
     times = []
     for step in range(a.warmup + a.steps):
         # each step a different bounded sample of the workload stream
@@ -217,7 +223,8 @@ def run_reference(a):
         "ms_per_step": round(tot / a.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"cfg2 sample: {n >> 20} MiB {a.cls} per step, C={C}",
-                   "chunk_size": C, "window": C, "min_match": 4, "max_match": 259},
+                   "chunk_size": C, "window": C, "min_match": 4, "max_match": 259,
+                   "parse": a.parse},
         "cpu_baseline": {"value": round(v, 6), "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": f"{n >> 20} MiB per step (chunks {n // C} per step), "
                                    "thread-per-chunk on all host cores"},
@@ -255,7 +262,7 @@ def run_dedup(a):
     if sharded:
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
-    p = lzr.Params(chunk_size=C)
+    p = lzr.Params(chunk_size=C, parse=PARSES[a.parse])
     n_glob = ((a.bytes_per_rank * world if a.bytes_per_rank else (16 << 30)) // C) * C
     N_glob = n_glob // C
     lo, hi = shard_range(N_glob, world, grank) if sharded else (0, N_glob)
@@ -367,7 +374,7 @@ def run_dedup(a):
         "data": "synthetic",
         "config": {"workload": workload, "global_bytes": n_glob, "unique_bytes": nub_all,
                    "dedup_ratio": round(n_glob / max(1, nub_all), 4), "chunk_size": C, "window": C,
-                   "min_match": 4, "max_match": 259,
+                   "min_match": 4, "max_match": 259, "parse": a.parse,
                    "parallelism": (f"dp{world}: contiguous chunk shards; global index by NCCL "
                                    "all-to-all to fingerprint owners; all-gather of totals")
                    if sharded else "1 GPU",
@@ -397,7 +404,7 @@ def run_dedup(a):
         fps = oracle.fingerprints(xs, C, n_threads=cores)
         ri, rh, _ = oracle.dedup_index(fps, 0)
         ub = np.concatenate([xs[i * C:(i + 1) * C] for i in np.flatnonzero(rh == 0)])
-        oracle.compress(ub, oracle.Params(chunk_size=C), n_threads=cores)
+        oracle.compress(ub, oracle.Params(chunk_size=C, parse=PARSES[a.parse]), n_threads=cores)
         dt = time.perf_counter() - tc
         ok = bool(np.array_equal(ri, idx[: smp // C].cpu().numpy().view(np.uint64)))
         line["cpu_baseline"] = {"value": round(ub.size / dt / 1e9, 6), "unit": UNIT, "cores": cores,
@@ -437,7 +444,7 @@ def main():
     if sharded:
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
-    p = lzr.Params(chunk_size=C)
+    p = lzr.Params(chunk_size=C, parse=PARSES[a.parse])
     # workload (BASELINE.json configs); weak = fixed bytes per GPU, strong = fixed total
     if a.config in (1, 4):
         scaling = "strong"
@@ -531,6 +538,8 @@ def main():
     achieved = enc_algo_bytes / enc_avg_s / 1e9
     if a.config == 2 and not a.bytes_per_rank:
         workload = f"cfg2: {n_rank >> 20} MiB {a.cls} per GPU, C=W={C}, m=4, M=259"
+        if a.parse != "greedy":
+            workload += f", {a.parse} parse"
     else:
         workload = (f"cfg{a.config}: {n_glob >> 20} MiB {a.cls} total ({scaling} scaling), "
                     f"C=W={C}, m=4, M=259")
@@ -542,7 +551,7 @@ def main():
         "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
         "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": C,
-                   "min_match": 4, "max_match": 259, "chunks_per_gpu": ws.N,
+                   "min_match": 4, "max_match": 259, "parse": a.parse, "chunks_per_gpu": ws.N,
                    "parallelism": f"dp{world} (contiguous chunk shards, NCCL all-gather of sizes)"
                    if sharded else "1 GPU",
                    "l2": (f"input ({n_rank >> 20} MiB/GPU) larger than L2 (126 MB); no flush"

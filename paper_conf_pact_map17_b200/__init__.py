@@ -27,6 +27,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("LZR_LIBRARY") or os.path.join(_PKG, "liblzr.so")
 
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CAPACITY, ERR_CUDA, ERR_CORRUPT = 0, -1, -2, -3, -4, -5
+PARSE_GREEDY, PARSE_LAZY = 0, 1  # lzr_params.parse (include/lzr.h; R8, R21)
 
 EXPORTED_SYMBOLS = [
     "lzr_validate_params", "lzr_num_chunks", "lzr_compress_bound", "lzr_compress_workspace_bytes",
@@ -48,7 +49,7 @@ class LzrError(RuntimeError):
 class _CParams(ctypes.Structure):
     _fields_ = [("chunk_size", ctypes.c_uint32), ("window", ctypes.c_uint32),
                 ("min_match", ctypes.c_uint32), ("max_match", ctypes.c_uint32),
-                ("tie_break", ctypes.c_uint32)]
+                ("tie_break", ctypes.c_uint32), ("parse", ctypes.c_uint32)]
 
 
 @dataclass(frozen=True)
@@ -59,11 +60,12 @@ class Params:
     min_match: int = 4
     max_match: int | None = None
     tie_break: int = 0
+    parse: int = 0  # PARSE_GREEDY (R8) or PARSE_LAZY (R21)
 
     def c(self) -> _CParams:
         w = self.chunk_size if self.window is None else self.window
         mm = self.min_match + 255 if self.max_match is None else self.max_match
-        return _CParams(self.chunk_size, w, self.min_match, mm, self.tie_break)
+        return _CParams(self.chunk_size, w, self.min_match, mm, self.tie_break, self.parse)
 
 
 _lib = None

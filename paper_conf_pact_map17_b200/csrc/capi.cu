@@ -104,6 +104,7 @@ int lzr_validate_params(const lzr_params* p) {
   if (p->min_match < 3 || p->min_match > 255) return LZR_ERR_INVALID_ARG;
   if (p->max_match < p->min_match || p->max_match > p->min_match + 255) return LZR_ERR_INVALID_ARG;
   if (p->tie_break != LZR_TIE_LONGEST_THEN_NEAREST) return LZR_ERR_UNSUPPORTED;
+  if (p->parse != LZR_PARSE_GREEDY && p->parse != LZR_PARSE_LAZY) return LZR_ERR_UNSUPPORTED;
   return LZR_OK;
 }
 
@@ -161,6 +162,7 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.W = p->window;
   a.m = p->min_match;
   a.M = p->max_match;
+  a.lazy = p->parse == LZR_PARSE_LAZY;
   a.kbytes = p->min_match < 4 ? p->min_match : 4;
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
   const uint32_t K = enc_warps_per_chunk(p->chunk_size);

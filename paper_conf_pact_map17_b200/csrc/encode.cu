@@ -226,8 +226,13 @@ __device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, u
 }
 
 // Returns (len << 16) | (0xFFFF - (d-1)), or 0 when no candidate reaches m.
+// floor > 0 (lazy parse only asks whether some match is longer than floor):
+// the generic path then evaluates only candidates that also match the byte at
+// offset floor; the result is exact whenever it exceeds floor (every candidate
+// reaching the maximum passes that test), otherwise it is some value <= floor.
 __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32_t n,
-                                               uint32_t nruns, const EncArgs& a, uint32_t lane) {
+                                               uint32_t nruns, const EncArgs& a, uint32_t lane,
+                                               uint32_t floor = 0) {
   const uint8_t* data = S.data;
   const uint32_t cap = min(a.M, n - p);  // p < n - m + 1  =>  cap >= m >= k
   const uint32_t kp = ld32u(data, p) & a.kmask;
@@ -240,7 +245,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   // are preloaded for the 16-byte compares.  (A separate path for lists of
   // <= 8 candidates -- 4-8 lanes per candidate -- and 64 candidates per round
   // both measured slower: mix 52.3 vs 51.0 / 51.5 GB/s.)
-  uint32_t best = 0, blen = 0;
+  uint32_t best = 0, blen = floor;
   const uint32_t rp = prun ? run_len(S.cb, p, cap) : 0u;
   uint32_t pw[4];
   {
@@ -283,7 +288,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
       if (l >= a.m) pk = (l << 16) | (0xFFFFu - (p - q - 1));
     }
     best = max(best, __reduce_max_sync(kFull, pk));
-    blen = best >> 16;
+    blen = max(floor, best >> 16);
     if (blen >= cap || lim < 32) break;
   }
   return best;
@@ -297,7 +302,11 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 // recorded.  A warp with a successor stops at the first of its token starts x
 // that the successor has recorded (x < prog[k+1]); sync[k] = x, or n if it ran
 // to the end.
-template <int K>
+// LZ (one-step lazy parse, R21): a match at q is taken only if the best match
+// at q + 1 is not strictly longer; otherwise q is a literal and the walk moves
+// to q + 1, whose best match is then already known (cached).  The decision at
+// q depends on q alone, so the meeting-point argument above is unchanged.
+template <int K, bool LZ>
 __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
                                              uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
                                              const EncArgs& a, uint32_t lane) {
@@ -308,6 +317,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
   uint32_t* sync = prog + K;
   uint32_t p = start, pub = start;
   uint32_t stop_at = n;
+  uint32_t cq = 0xFFFFFFFFu, cr = 0;  // LZ: best match already computed at cq
 #ifdef LZR_PHASE_TIMING
   long long t_bm = 0, n_bm = 0, n_it = 0;
 #endif
@@ -331,12 +341,19 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
 #ifdef LZR_PHASE_TIMING
       const long long tb0 = clock64();
 #endif
-      r = best_match(S, q, n, nruns, a, lane);
+      r = (LZ && q == cq) ? cr : best_match(S, q, n, nruns, a, lane);
 #ifdef LZR_PHASE_TIMING
       t_bm += clock64() - tb0;
       ++n_bm;
 #endif
-      const uint32_t l = r >> 16;
+      uint32_t l = r >> 16;
+      // LZ: a longer match at q + 1 is possible only if l is below its cap
+      // min(M, n - q - 1) and q + 1 has a same-key candidate
+      if (LZ && l >= a.m && l < min(a.M, n - q - 1) && ((S.cand[(q + 1) >> 5] >> ((q + 1) & 31u)) & 1u)) {
+        cr = best_match(S, q + 1, n, nruns, a, lane, l);  // exact if > l
+        cq = q + 1;
+        if ((cr >> 16) > l) l = 0;  // deferred: x[q] is a literal
+      }
       tok_len = l >= a.m ? l : 1u;
       cnt = L + 1;  // <= 32
     }
@@ -448,7 +465,7 @@ struct MinBlocks {
   static constexpr int value = K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1);
 };
 
-template <int K, int NS>
+template <int K, int NS, bool LZ>
 __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
     lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
@@ -739,7 +756,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
       // density growing ~linearly with the position (walk_bound)
       const uint32_t start = walk_bound(n, k, K), nb = walk_bound(n, k + 1, K);
       if (start < n && (k == 0 || start > 0))
-        walk_segment<K>(S, d1, k, start, nb, n, P, nruns, a, lane);
+        walk_segment<K, LZ>(S, d1, k, start, nb, n, P, nruns, a, lane);
     }
     GSYNC(7);
 
@@ -897,7 +914,7 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
   }
 }
 
-template <int K, int NS>
+template <int K, int NS, bool LZ>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
   const int max_groups = MaxThreads<K>::value / (32 * K);
@@ -905,20 +922,20 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   if (groups > 15) groups = 15;  // named barriers 1..15
   if (groups < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)groups * a.L.per_group;
-  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS>,
+  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
   int per_sm = 1;
   if (MinBlocks<K>::value > 1 &&
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS>,
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ>,
                                                     groups * 32 * K, smem) != cudaSuccess)
     per_sm = 1;
   if (per_sm < 1) per_sm = 1;
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
-  lzr_encode_kernel<K, NS><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS, LZ><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -933,29 +950,37 @@ extern "C" int lzr_debug_phase_times(unsigned long long* out) {
 }
 #endif
 
-cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s,
-                          int* launches) {
+namespace {
+template <bool LZ>
+cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   switch (a.L.K) {
-    case 1: return launch_k<1, 1>(a, sm_count, smem_optin, s, launches);
-    case 2: return launch_k<2, 1>(a, sm_count, smem_optin, s, launches);
-    case 3: return launch_k<3, 1>(a, sm_count, smem_optin, s, launches);
+    case 1: return launch_k<1, 1, LZ>(a, sm_count, smem_optin, s, launches);
+    case 2: return launch_k<2, 1, LZ>(a, sm_count, smem_optin, s, launches);
+    case 3: return launch_k<3, 1, LZ>(a, sm_count, smem_optin, s, launches);
     case 4:
       switch (a.L.nsplit) {
-        case 1: return launch_k<4, 1>(a, sm_count, smem_optin, s, launches);
-        case 2: return launch_k<4, 2>(a, sm_count, smem_optin, s, launches);
-        case 4: return launch_k<4, 4>(a, sm_count, smem_optin, s, launches);
+        case 1: return launch_k<4, 1, LZ>(a, sm_count, smem_optin, s, launches);
+        case 2: return launch_k<4, 2, LZ>(a, sm_count, smem_optin, s, launches);
+        case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;
       }
     case 8:
       switch (a.L.nsplit) {
-        case 1: return launch_k<8, 1>(a, sm_count, smem_optin, s, launches);
-        case 2: return launch_k<8, 2>(a, sm_count, smem_optin, s, launches);
-        case 4: return launch_k<8, 4>(a, sm_count, smem_optin, s, launches);
-        case 8: return launch_k<8, 8>(a, sm_count, smem_optin, s, launches);
+        case 1: return launch_k<8, 1, LZ>(a, sm_count, smem_optin, s, launches);
+        case 2: return launch_k<8, 2, LZ>(a, sm_count, smem_optin, s, launches);
+        case 4: return launch_k<8, 4, LZ>(a, sm_count, smem_optin, s, launches);
+        case 8: return launch_k<8, 8, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;
       }
     default: return cudaErrorInvalidConfiguration;
   }
+}
+}  // namespace
+
+cudaError_t launch_encode(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s,
+                          int* launches) {
+  return a.lazy ? launch_kns<true>(a, sm_count, smem_optin, s, launches)
+                : launch_kns<false>(a, sm_count, smem_optin, s, launches);
 }
 
 }  // namespace lzr

@@ -141,6 +141,7 @@ struct EncArgs {
   size_t n_bytes;
   uint32_t N;  // chunks (fits: N <= 2^32 - 1 checked on host)
   uint32_t C, W, m, M;
+  uint32_t lazy;           // parse rule: 0 greedy (R8), 1 one-step lazy (R21)
   uint32_t kbytes, kmask;  // candidate key = first min(m,4) bytes
   EncLayout L;
   uint8_t* slots;    // workspace: chunk i's stream at slots + i*C

@@ -90,6 +90,9 @@ def test_host_argument_errors(lzr):
                                  ctypes.c_void_p(256), 4096, ctypes.c_void_p(256),
                                  ctypes.c_void_p(256), None, ctypes.c_void_p(256), 1 << 20,
                                  None) == lzr.ERR_UNSUPPORTED
+    # parse rule: greedy (0) and lazy (1) are valid, anything else is unsupported
+    assert L.lzr_validate_params(ctypes.byref(lzr.Params(parse=lzr.PARSE_LAZY).c())) == lzr.OK
+    assert L.lzr_validate_params(ctypes.byref(lzr.Params(parse=2).c())) == lzr.ERR_UNSUPPORTED
     # n == 0 is a no-op
     assert L.lzr_compress_encode(None, 0, cp, None, None, 0, None) == lzr.OK
 

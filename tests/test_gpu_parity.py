@@ -29,7 +29,7 @@ def lzr():
 
 def _ref_params(ref, p):
     return ref.Params(chunk_size=p.chunk_size, window=p.window, min_match=p.min_match,
-                      max_match=p.max_match)
+                      max_match=p.max_match, parse=p.parse)
 
 
 def _gpu_compress(lzr, x: np.ndarray, p):
@@ -127,12 +127,14 @@ def test_batch_edges(lzr, ref, nchunks):
 
 def test_golden_through_gpu(lzr, ref):
     import json, os
-    path = os.path.join(os.path.dirname(__file__), "golden", "appendix_a.jsonl")
-    for line in open(path):
+    lines = []
+    for f in ("appendix_a.jsonl", "lazy_examples.jsonl"):
+        lines += open(os.path.join(os.path.dirname(__file__), "golden", f)).readlines()
+    for line in lines:
         c = json.loads(line)
         pp = c["params"]
         p = lzr.Params(chunk_size=pp["chunk_size"], window=pp["window"], min_match=pp["min_match"],
-                       max_match=pp["max_match"])
+                       max_match=pp["max_match"], parse=pp.get("parse", 0))
         if "input_ascii" in c:
             x = np.frombuffer(c["input_ascii"].encode(), np.uint8).copy()
         else:
