@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-decode", action="store_true")
+    ap.add_argument("--window", type=int, default=None,
+                    help="W < C (SURVEY.md §8(f) N4); default W = C (the configs)")
     ap.add_argument("--parse", default="greedy", choices=["greedy", "lazy"],
                     help="parse rule (DESIGN.md R8 greedy, R21 one-step lazy; SURVEY.md §8(f) N4)")
     return ap.parse_args()
@@ -177,7 +179,8 @@ def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
     xs = x_host[: nchunks * C]
     cores = len(os.sched_getaffinity(0))
     t0 = time.perf_counter()
-    r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, oracle.Params(chunk_size=C, parse=p_gpu.parse),
+    r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, oracle.Params(chunk_size=C, window=p_gpu.window,
+                                                                  parse=p_gpu.parse),
                                                    n_threads=cores)
     dt = time.perf_counter() - t0
     ok = bool(np.array_equal(r_sizes, g_sizes[:nchunks]) and np.array_equal(r_offs, g_offs[:nchunks])
@@ -189,6 +192,32 @@ def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
 
 
 PARSES = {"greedy": 0, "lazy": 1}  # lzr_params.parse (include/lzr.h)
+
+
+def cpu_fast(x_host, p_gpu, g_sizes, g_out):
+    """the fast exact CPU compressor (cpuref/, hash chains +
+    run-aware search, thread-per-chunk on all host cores, §3.2(1)) on the
+    whole timed stream -- the CPU arm of the paper's GPU-usage decision (P:16
+    §3.2(3)) -- with every chunk checked against the GPU output."""
+    import numpy as np
+
+    import cpuref
+
+    cores = len(os.sched_getaffinity(0))
+    cp = cpuref.Params(chunk_size=p_gpu.chunk_size, window=p_gpu.window, parse=p_gpu.parse)
+    slots = np.empty(x_host.size, np.uint8)
+    cpuref.compress(x_host[: 64 * p_gpu.chunk_size], cp, n_threads=cores)  # warm-up (build, pages)
+    best = None
+    for _ in range(2):
+        t0 = time.perf_counter()
+        out, sizes, _, tot = cpuref.compress(x_host, cp, n_threads=cores, slots=slots)
+        dt = time.perf_counter() - t0
+        best = dt if best is None else min(best, dt)
+    ok = bool(np.array_equal(sizes, g_sizes) and np.array_equal(out, g_out))
+    return {"value": round(x_host.size / best / 1e9, 4), "unit": UNIT, "cores": cores,
+            "kind": "fast exact CPU compressor (cpuref/: hash chains + run-aware search, pinned to the oracle)",
+            "sample": f"the whole timed stream ({x_host.size >> 20} MiB), best of 2",
+            "parity_vs_gpu": "bit-exact, every chunk" if ok else "MISMATCH"}
 
 
 def run_reference(a):
@@ -204,7 +233,7 @@ def run_reference(a):
     C = a.chunk_size
     cores = len(os.sched_getaffinity(0))
     n = (a.ref_sample_bytes // C) * C
-    p = oracle.Params(chunk_size=C, parse=PARSES[a.parse])
+    p = oracle.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse])
     times = []
     for step in range(a.warmup + a.steps):
         # each step a different bounded sample of the workload stream
@@ -223,7 +252,7 @@ def run_reference(a):
         "ms_per_step": round(tot / a.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"cfg2 sample: {n >> 20} MiB {a.cls} per step, C={C}",
-                   "chunk_size": C, "window": C, "min_match": 4, "max_match": 259,
+                   "chunk_size": C, "window": a.window or C, "min_match": 4, "max_match": 259,
                    "parse": a.parse},
         "cpu_baseline": {"value": round(v, 6), "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": f"{n >> 20} MiB per step (chunks {n // C} per step), "
@@ -262,7 +291,7 @@ def run_dedup(a):
     if sharded:
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
-    p = lzr.Params(chunk_size=C, parse=PARSES[a.parse])
+    p = lzr.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse])
     n_glob = ((a.bytes_per_rank * world if a.bytes_per_rank else (16 << 30)) // C) * C
     N_glob = n_glob // C
     lo, hi = shard_range(N_glob, world, grank) if sharded else (0, N_glob)
@@ -373,7 +402,7 @@ def run_dedup(a):
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
         "config": {"workload": workload, "global_bytes": n_glob, "unique_bytes": nub_all,
-                   "dedup_ratio": round(n_glob / max(1, nub_all), 4), "chunk_size": C, "window": C,
+                   "dedup_ratio": round(n_glob / max(1, nub_all), 4), "chunk_size": C, "window": a.window or C,
                    "min_match": 4, "max_match": 259, "parse": a.parse,
                    "parallelism": (f"dp{world}: contiguous chunk shards; global index by NCCL "
                                    "all-to-all to fingerprint owners; all-gather of totals")
@@ -404,7 +433,8 @@ def run_dedup(a):
         fps = oracle.fingerprints(xs, C, n_threads=cores)
         ri, rh, _ = oracle.dedup_index(fps, 0)
         ub = np.concatenate([xs[i * C:(i + 1) * C] for i in np.flatnonzero(rh == 0)])
-        oracle.compress(ub, oracle.Params(chunk_size=C, parse=PARSES[a.parse]), n_threads=cores)
+        oracle.compress(ub, oracle.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse]),
+                        n_threads=cores)
         dt = time.perf_counter() - tc
         ok = bool(np.array_equal(ri, idx[: smp // C].cpu().numpy().view(np.uint64)))
         line["cpu_baseline"] = {"value": round(ub.size / dt / 1e9, 6), "unit": UNIT, "cores": cores,
@@ -444,7 +474,7 @@ def main():
     if sharded:
         dist.init_process_group("nccl", device_id=dev)
     C = a.chunk_size
-    p = lzr.Params(chunk_size=C, parse=PARSES[a.parse])
+    p = lzr.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse])
     # workload (BASELINE.json configs); weak = fixed bytes per GPU, strong = fixed total
     if a.config in (1, 4):
         scaling = "strong"
@@ -540,9 +570,13 @@ def main():
         workload = f"cfg2: {n_rank >> 20} MiB {a.cls} per GPU, C=W={C}, m=4, M=259"
         if a.parse != "greedy":
             workload += f", {a.parse} parse"
+        if a.window and a.window != C:
+            workload += f", W={a.window}"
     else:
         workload = (f"cfg{a.config}: {n_glob >> 20} MiB {a.cls} total ({scaling} scaling), "
                     f"C=W={C}, m=4, M=259")
+        if a.parse != "greedy" or (a.window and a.window != C):
+            workload += f", W={a.window or C}, {a.parse} parse"
     traffic = traffic_from_profiles(workload)
 
     line = {
@@ -550,7 +584,7 @@ def main():
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 4),
         "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u8",
         "data": "synthetic",
-        "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": C,
+        "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": a.window or C,
                    "min_match": 4, "max_match": 259, "parse": a.parse, "chunks_per_gpu": ws.N,
                    "parallelism": f"dp{world} (contiguous chunk shards, NCCL all-gather of sizes)"
                    if sharded else "1 GPU",
@@ -631,6 +665,20 @@ def main():
         g_out = ws.out[:end].cpu().numpy()
         line["cpu_baseline"] = cpu_baseline(x[:smp].cpu().numpy(), p, sizes[:ns], g_offs, g_out,
                                             smp)
+    if rank == 0 and not a.no_cpu and not a.bytes_per_rank and a.config in (1, 2, 3):
+        g_all = ws.out[:total].cpu().numpy()
+        line["cpu_fast"] = cpu_fast(x.cpu().numpy(), p, sizes, g_all)
+        # the paper's GPU-usage decision (§3.2(3) "we compare the compression
+        # performance of the CPU and the GPU to determine when to use the GPU"),
+        # from this run's measured numbers
+        gpu_v = line["value"]
+        e2e_v = line.get("e2e", {}).get("value")
+        cpu_v = line["cpu_fast"]["value"]
+        line["integration"] = {
+            "gpu_device_gbs": gpu_v, "gpu_e2e_gbs": e2e_v, "cpu_fast_gbs": cpu_v,
+            "gpu_over_cpu_e2e": round(e2e_v / cpu_v, 2) if e2e_v else None,
+            "use_gpu_for_compression": bool((e2e_v or gpu_v) > cpu_v),
+            "paper": "GPU 88.3% better than CPU (P:16 §3.2(3), other hardware; context)"}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if sharded:

@@ -1,14 +1,17 @@
 """Full-size parity at BASELINE.json's configs 3, 4 and 5 in the launch
 configuration bench.py times (one GPU): deterministic chunk samples against the
-oracle, and properties that hold at any size (offsets = exclusive scan of
-sizes, full GPU round trip; for the dedup stream, every index number equals the
-generator's ground-truth source chunk and its fingerprint matches)."""
+oracle, EVERY chunk against the fast exact CPU compressor (cpuref/, itself
+pinned to the oracle by tests/test_cpuref.py), and properties that hold at any
+size (offsets = exclusive scan of sizes, full GPU round trip; for the dedup
+stream, every index number equals the generator's ground-truth source chunk and
+its fingerprint matches)."""
 import numpy as np
 import pytest
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
+import cpuref  # noqa: E402
 import synth  # noqa: E402
 
 
@@ -23,7 +26,28 @@ def lzr():
     return m
 
 
-def _sampled_check(lzr, ref, xd, C, every, roundtrip=True):
+def _full_stream_check(xd, C, out, sizes, offs, parse=0, batch=256 << 20):
+    """Every chunk, batch by batch: sizes and the compacted bytes of the batch
+    equal cpuref's (= the oracle's definition) exactly."""
+    n = xd.numel()
+    N = -(-n // C)
+    g_sizes = sizes.cpu().numpy().view(np.uint32)
+    g_offs = offs.cpu().numpy().view(np.uint64)
+    per = max(1, batch // C)
+    slots = np.empty(per * C, np.uint8)
+    for i0 in range(0, N, per):
+        i1 = min(N, i0 + per)
+        xs = xd[i0 * C: min(n, i1 * C)].cpu().numpy()
+        c_out, c_sizes, _, c_tot = cpuref.compress(xs, cpuref.Params(chunk_size=C, parse=parse), slots=slots)
+        assert np.array_equal(g_sizes[i0:i1], c_sizes), i0
+        lo = int(g_offs[i0])
+        got = out[lo: lo + int(c_tot)].cpu().numpy()
+        if not np.array_equal(got, c_out):
+            bad = int(np.argmax(got != c_out))
+            raise AssertionError(f"batch at chunk {i0}: first differing byte {bad}")
+
+
+def _sampled_check(lzr, ref, xd, C, every, roundtrip=True, full=True):
     n = xd.numel()
     p = lzr.Params(chunk_size=C)
     out, sizes, offs, total = lzr.compress(xd, p)
@@ -41,6 +65,8 @@ def _sampled_check(lzr, ref, xd, C, every, roundtrip=True):
         assert got == r_streams[k], i
     assert g_offs[0] == 0 and np.array_equal(g_offs[1:], np.cumsum(g_sizes[:-1], dtype=np.uint64))
     assert int(total.item()) == int(g_sizes.sum(dtype=np.uint64))
+    if full:
+        _full_stream_check(xd, C, out, sizes, offs)
     if roundtrip:
         y, err = lzr.decompress(out, sizes, offs, n, p)
         torch.cuda.synchronize()
@@ -54,6 +80,16 @@ def test_config3_1gib_sampled(lzr, ref, C):
     xd = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
     synth.fill_device(xd, C, "mix")
     _sampled_check(lzr, ref, xd, C, every=1024 if C >= 16384 else 256)
+
+
+def test_config3_1gib_lazy_full_stream(lzr):
+    """The lazy parse (R21) over the whole 1 GiB mix stream, every chunk."""
+    xd = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+    synth.fill_device(xd, 4096, "mix")
+    p = lzr.Params(parse=lzr.PARSE_LAZY)
+    out, sizes, offs, total = lzr.compress(xd, p)
+    torch.cuda.synchronize()
+    _full_stream_check(xd, 4096, out, sizes, offs, parse=1)
 
 
 def test_config4_16gib_sampled(lzr, ref):
