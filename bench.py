@@ -608,6 +608,26 @@ def main():
                         torch.cuda.get_device_properties(dev).multi_processor_count)
     if lim:
         line["roofline"]["limiter"] = lim
+    # the shared-memory side of the roofline.  (1) the encode
+    # kernel's measured shared-memory pipe utilisation (ncu capture of the same
+    # workload); (2) the exhaustive byte-compare ceiling -- one shared-memory
+    # byte per (p, d) cell, (C-1)/2 cells per input byte, 148 SMs x 128 B/clk at
+    # the sampled clock -- which the token-start-only, candidate-exact search is
+    # not bound by (ratio > 1 = faster than any cell-by-cell search could be).
+    ent = _profile_entry(workload)
+    sm_mhz = line["clocks"].get("sm_mhz")
+    n_sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    if sm_mhz:
+        smem_peak = n_sms * 128 * float(sm_mhz) * 1e6
+        ceil_gbs = smem_peak / ((C - 1) / 2) / 1e9 * world
+        line["roofline"]["smem"] = {
+            "pipe_frac": round(ent["smem_pipe_pct"] / 100, 4) if ent and ent.get("smem_pipe_pct") else None,
+            "pipe_source": ent.get("source") if ent else None,
+            "peak_TBps": round(smem_peak / 1e12, 2),
+            "exhaustive_ceiling_gbs": round(ceil_gbs, 3),
+            "value_over_exhaustive_ceiling": round(value / ceil_gbs, 3)}
+        if ent and ent.get("stall_share"):
+            line["roofline"]["stalls"] = ent["stall_share"]
 
     # ---- decompression of the same batch, output GB/s
     if not a.no_decode:

@@ -53,6 +53,8 @@ summ[workload] = {"round": R, "dram_bytes_per_launch": full["dram_bytes_per_laun
                   "duration_s": full.get("gpu__time_duration.sum"),
                   "warp_inst_per_launch": full.get("smsp__inst_executed.sum"),
                   "ipc": full.get("sm__inst_executed.avg.per_cycle_active"),
+                  "smem_pipe_pct": full.get("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed"),
+                  "stall_share": full.get("stall_share"),
                   "source": f"profiles/ncu_{R}.json (ncu --set full, one encode launch of bench.py)"}
 json.dump(summ, open(summ_path, "w"), indent=1)
 json.dump(out, open(os.path.join(ROOT, "profiles", f"ncu_{R}.json"), "w"), indent=1)

@@ -17,9 +17,10 @@ ap.add_argument("--mib", type=int, default=64)
 ap.add_argument("--iters", type=int, default=2)
 ap.add_argument("--chunk-size", type=int, default=4096)
 ap.add_argument("--decode", action="store_true")
+ap.add_argument("--parse", type=int, default=0)  # 0 greedy, 1 lazy (R21)
 a = ap.parse_args()
 n = a.mib << 20
-p = lzr.Params(chunk_size=a.chunk_size)
+p = lzr.Params(chunk_size=a.chunk_size, parse=a.parse)
 x = torch.empty(n, dtype=torch.uint8, device="cuda")
 synth.fill_device(x, a.chunk_size, a.cls)
 ws = lzr.Workspace(n, p, x.device)
