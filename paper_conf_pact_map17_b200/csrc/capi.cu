@@ -428,6 +428,15 @@ int host_sets() {  // LZR_HOST_SETS=2..8 overrides (tuning)
   return v;
 }
 
+bool host_split() {  // LZR_HOST_SPLIT=0 puts the H2D back on the set's compute stream (A/B)
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("LZR_HOST_SPLIT");
+    v = (e && *e == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+
 size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
   if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
   return host_sets() * align_up_z(set_bytes(batch_bytes, p), 256);
@@ -453,14 +462,42 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   const int kHostSets = host_sets();
   if (scratch_bytes < kHostSets * per) return LZR_ERR_CAPACITY;
   HostSet set[kMaxHostSets];
-  cudaStream_t s[kMaxHostSets];
+  cudaStream_t s[kMaxHostSets], cin[kMaxHostSets];
+  cudaEvent_t ev_in[kMaxHostSets], ev_kdone[kMaxHostSets];
+  // split (default): a set's H2D runs on its own copy stream and waits only for
+  // the kernels of the set's previous batch (its input buffer), not for that
+  // batch's D2H of compressed bytes (which reads the output buffer)
+  const bool split = host_split();
   int made = 0;
   for (; made < kHostSets; ++made) {
     set[made] = carve((uint8_t*)d_scratch + made * per, batch_bytes, p);
     if (cudaStreamCreateWithFlags(&s[made], cudaStreamNonBlocking) != cudaSuccess) break;
+    if (cudaStreamCreateWithFlags(&cin[made], cudaStreamNonBlocking) != cudaSuccess) {
+      cudaStreamDestroy(s[made]);
+      break;
+    }
+    if (cudaEventCreateWithFlags(&ev_in[made], cudaEventDisableTiming) != cudaSuccess) {
+      cudaStreamDestroy(s[made]);
+      cudaStreamDestroy(cin[made]);
+      break;
+    }
+    if (cudaEventCreateWithFlags(&ev_kdone[made], cudaEventDisableTiming) != cudaSuccess) {
+      cudaStreamDestroy(s[made]);
+      cudaStreamDestroy(cin[made]);
+      cudaEventDestroy(ev_in[made]);
+      break;
+    }
   }
+  auto destroy = [&](int k) {
+    for (int i = 0; i < k; ++i) {
+      cudaStreamDestroy(s[i]);
+      cudaStreamDestroy(cin[i]);
+      cudaEventDestroy(ev_in[i]);
+      cudaEventDestroy(ev_kdone[i]);
+    }
+  };
   if (made < kHostSets) {
-    for (int i = 0; i < made; ++i) cudaStreamDestroy(s[i]);
+    destroy(made);
     return LZR_ERR_CUDA;
   }
   const size_t nb = (n_bytes + batch_bytes - 1) / batch_bytes;
@@ -475,12 +512,22 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
     const size_t len = n_bytes - lo < batch_bytes ? n_bytes - lo : batch_bytes;
     const size_t c0 = b * chunks_per_batch;
     const size_t N = (len + C - 1) / C;
-    if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, ss) != cudaSuccess)
+    const int k = (int)(b % kHostSets);
+    if (split) {
+      // h.in is free once the kernels of this set's previous batch are done
+      if (b >= (size_t)kHostSets && cudaStreamWaitEvent(cin[k], ev_kdone[k], 0) != cudaSuccess)
+        return LZR_ERR_CUDA;
+      if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, cin[k]) != cudaSuccess ||
+          cudaEventRecord(ev_in[k], cin[k]) != cudaSuccess || cudaStreamWaitEvent(ss, ev_in[k], 0) != cudaSuccess)
+        return LZR_ERR_CUDA;
+    } else if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, ss) != cudaSuccess) {
       return LZR_ERR_CUDA;
+    }
     int r = lzr_compress_chunks(h.in, len, p, h.out, batch_bytes, h.sizes, h.offs, h.total, h.ws,
                                 h.ws_bytes, (lzr_stream_t)ss);
     if (r) return r;
     launches += t_launches;
+    if (split && cudaEventRecord(ev_kdone[k], ss) != cudaSuccess) return LZR_ERR_CUDA;
     if (cudaMemcpyAsync(h_sizes + c0, h.sizes, 4 * N, cudaMemcpyDeviceToHost, ss) != cudaSuccess ||
         cudaMemcpyAsync(h_offsets + c0, h.offs, 8 * N, cudaMemcpyDeviceToHost, ss) != cudaSuccess)
       return LZR_ERR_CUDA;
@@ -512,8 +559,10 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   for (size_t b = nb > kHostSets - 1 ? nb - (kHostSets - 1) : 0; b < nb && rc == LZR_OK; ++b)
     rc = finish(b);
   for (int i = 0; i < kHostSets; ++i)
-    if (cudaStreamSynchronize(s[i]) != cudaSuccess && rc == LZR_OK) rc = LZR_ERR_CUDA;
-  for (int i = 0; i < kHostSets; ++i) cudaStreamDestroy(s[i]);
+    if ((cudaStreamSynchronize(s[i]) != cudaSuccess || cudaStreamSynchronize(cin[i]) != cudaSuccess) &&
+        rc == LZR_OK)
+      rc = LZR_ERR_CUDA;
+  destroy(kHostSets);
   if (h_total) *h_total = running;
   t_launches = launches;
   return rc;

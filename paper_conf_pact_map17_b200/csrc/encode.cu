@@ -455,18 +455,26 @@ __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
 #ifndef LZR_K8_MINB
 #define LZR_K8_MINB 1
 #endif
-template <int K>
+// G1: one group per CTA (K = 4 only; 9 CTAs of 4 warps per SM, same registers
+// and occupancy).  Used for launches of few waves: a CTA then leaves the SM as
+// soon as its one group runs out of chunks, so the tail of the launch (the last
+// chunks, up to one chunk latency) overlaps the next launch on another stream
+// instead of holding the SM (1 x B200, 16 MiB batches on 4 streams: 46.6 ->
+// 50.8 GB/s; one 256 MiB launch: 51.9 -> 50.5, so large launches keep 3 x 3).
+template <int K, bool G1 = false>
 struct MaxThreads {
   static constexpr int value =
-      K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : LZR_K8_THREADS)));
+      G1 ? 32 * K
+         : (K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : LZR_K8_THREADS))));
 };
-template <int K>
+template <int K, bool G1 = false>
 struct MinBlocks {
-  static constexpr int value = K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1);
+  static constexpr int value = G1 ? (K == 4 ? 9 : 1) : (K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1));
 };
+constexpr uint32_t kG1MaxWaves = 12;  // launches of fewer chunk waves than this use G1
 
-template <int K, int NS, bool LZ>
-__global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
+template <int K, int NS, bool LZ, bool G1>
+__global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::value)
     lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
@@ -914,28 +922,28 @@ __global__ void __launch_bounds__(MaxThreads<K>::value, MinBlocks<K>::value)
   }
 }
 
-template <int K, int NS, bool LZ>
+template <int K, int NS, bool LZ, bool G1 = false>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
-  const int max_groups = MaxThreads<K>::value / (32 * K);
+  const int max_groups = MaxThreads<K, G1>::value / (32 * K);
   if (groups > max_groups) groups = max_groups;
   if (groups > 15) groups = 15;  // named barriers 1..15
   if (groups < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)groups * a.L.per_group;
-  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ>,
+  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (err != cudaSuccess) return err;
   // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
   int per_sm = 1;
-  if (MinBlocks<K>::value > 1 &&
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ>,
+  if (MinBlocks<K, G1>::value > 1 &&
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1>,
                                                     groups * 32 * K, smem) != cudaSuccess)
     per_sm = 1;
   if (per_sm < 1) per_sm = 1;
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
-  lzr_encode_kernel<K, NS, LZ><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS, LZ, G1><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -959,7 +967,11 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
     case 3: return launch_k<3, 1, LZ>(a, sm_count, smem_optin, s, launches);
     case 4:
       switch (a.L.nsplit) {
-        case 1: return launch_k<4, 1, LZ>(a, sm_count, smem_optin, s, launches);
+        case 1:
+          // few waves of chunks: one group per CTA (see MaxThreads)
+          if (a.N < kG1MaxWaves * 9u * (uint32_t)sm_count)
+            return launch_k<4, 1, LZ, true>(a, sm_count, smem_optin, s, launches);
+          return launch_k<4, 1, LZ>(a, sm_count, smem_optin, s, launches);
         case 2: return launch_k<4, 2, LZ>(a, sm_count, smem_optin, s, launches);
         case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;

@@ -8,7 +8,7 @@ import synth, paper_conf_pact_map17_b200 as lzr
 n = 256 << 20
 p = lzr.Params()
 x = torch.empty(n, dtype=torch.uint8, device="cuda"); synth.fill_device(x, 4096, "mix")
-for mb in [256, 64, 32, 16, 8]:
+for mb in [int(v) for v in (sys.argv[1] if len(sys.argv) > 1 else "256,64,32,16,8").split(",")]:
     b = mb << 20
     k = n // b
     for ns in (1, 4):
