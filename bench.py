@@ -673,7 +673,7 @@ def main():
             e2e_v = n_e2e * world / float(tt.item()) / 1e9
         line["e2e"] = {"value": round(e2e_v, 4), "unit": UNIT, "h2d_bytes_per_step": n_e2e,
                        "d2h_bytes_per_step": int(tot) + 12 * n_e2e_chunks,
-                       "api": "lzr_compress_host (pinned host in/out, 16 MiB batches, 4 streams)"
+                       "api": "lzr_compress_host (pinned host in/out, 16 MiB batches, 3 buffer sets, shared H2D / D2H copy streams)"
                               + ("" if n_e2e == n_rank else f", first {n_e2e >> 20} MiB per GPU")}
         del scratch
 

@@ -417,24 +417,31 @@ HostSet carve(uint8_t* base, size_t batch, const lzr_params* p) {
 // (H2D); a set is reused only after its D2H was issued on its own stream
 // (stream order).
 constexpr int kMaxHostSets = 8;
-// default 4 sets (e2e sweep on 1 x B200, 256 MiB mix, PCIe 55 GB/s one way / 94
-// both ways: 3 sets x 32 MiB 31.1 GB/s, 4 x 16 MiB 35.7, 6 x 16 MiB 32.6)
+// default 3 sets with shared copy streams (e2e sweep on 1 x B200, 256 MiB mix,
+// PCIe 55 GB/s one way / 93 both ways, tools/e2e_sweep.py; 8/16/32 MiB batches):
+// 3 sets 33.8/39.5/37.1 GB/s, 4 sets 37.6/38.6/36.4, 6 sets 35.6/36.0/32.6; a
+// copy stream per set 33.0/37.4/37.0 (3 sets); H2D on the compute stream
+// 32.6/37.0/36.5 (4 sets).  More sets split the link and the SMs over more
+// batches at once, so each batch's bytes arrive later
 int host_sets() {  // LZR_HOST_SETS=2..8 overrides (tuning)
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("LZR_HOST_SETS");
-    v = (e && *e >= '2' && *e <= '8') ? (*e - '0') : 4;
+    v = (e && *e >= '2' && *e <= '8') ? (*e - '0') : 3;
   }
   return v;
 }
 
-bool host_split() {  // LZR_HOST_SPLIT=0 puts the H2D back on the set's compute stream (A/B)
+// copy-stream mode (LZR_HOST_SPLIT overrides, A/B): 0 = H2D on the set's
+// compute stream; 1 = H2D on a copy stream per set; 2 = one H2D stream and one
+// D2H stream shared by all sets (copies in batch order at full link rate)
+int host_split() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("LZR_HOST_SPLIT");
-    v = (e && *e == '0') ? 0 : 1;
+    v = (e && *e >= '0' && *e <= '2') ? (*e - '0') : 2;
   }
-  return v == 1;
+  return v;
 }
 
 size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
@@ -463,11 +470,12 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   if (scratch_bytes < kHostSets * per) return LZR_ERR_CAPACITY;
   HostSet set[kMaxHostSets];
   cudaStream_t s[kMaxHostSets], cin[kMaxHostSets];
-  cudaEvent_t ev_in[kMaxHostSets], ev_kdone[kMaxHostSets];
-  // split (default): a set's H2D runs on its own copy stream and waits only for
-  // the kernels of the set's previous batch (its input buffer), not for that
-  // batch's D2H of compressed bytes (which reads the output buffer)
-  const bool split = host_split();
+  cudaEvent_t ev_in[kMaxHostSets], ev_kdone[kMaxHostSets], ev_out[kMaxHostSets];
+  // split (mode >= 1): a set's H2D waits only for the kernels of the set's
+  // previous batch (its input buffer), not for that batch's D2H of compressed
+  // bytes (which reads the output buffer; mode 2: the kernels wait for that)
+  const int mode = host_split();
+  const bool split = mode >= 1;
   int made = 0;
   for (; made < kHostSets; ++made) {
     set[made] = carve((uint8_t*)d_scratch + made * per, batch_bytes, p);
@@ -487,6 +495,13 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
       cudaEventDestroy(ev_in[made]);
       break;
     }
+    if (cudaEventCreateWithFlags(&ev_out[made], cudaEventDisableTiming) != cudaSuccess) {
+      cudaStreamDestroy(s[made]);
+      cudaStreamDestroy(cin[made]);
+      cudaEventDestroy(ev_in[made]);
+      cudaEventDestroy(ev_kdone[made]);
+      break;
+    }
   }
   auto destroy = [&](int k) {
     for (int i = 0; i < k; ++i) {
@@ -494,6 +509,7 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
       cudaStreamDestroy(cin[i]);
       cudaEventDestroy(ev_in[i]);
       cudaEventDestroy(ev_kdone[i]);
+      cudaEventDestroy(ev_out[i]);
     }
   };
   if (made < kHostSets) {
@@ -514,11 +530,15 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
     const size_t N = (len + C - 1) / C;
     const int k = (int)(b % kHostSets);
     if (split) {
+      cudaStream_t cs = mode == 2 ? cin[0] : cin[k];
       // h.in is free once the kernels of this set's previous batch are done
-      if (b >= (size_t)kHostSets && cudaStreamWaitEvent(cin[k], ev_kdone[k], 0) != cudaSuccess)
+      if (b >= (size_t)kHostSets && cudaStreamWaitEvent(cs, ev_kdone[k], 0) != cudaSuccess)
         return LZR_ERR_CUDA;
-      if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, cin[k]) != cudaSuccess ||
-          cudaEventRecord(ev_in[k], cin[k]) != cudaSuccess || cudaStreamWaitEvent(ss, ev_in[k], 0) != cudaSuccess)
+      if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, cs) != cudaSuccess ||
+          cudaEventRecord(ev_in[k], cs) != cudaSuccess || cudaStreamWaitEvent(ss, ev_in[k], 0) != cudaSuccess)
+        return LZR_ERR_CUDA;
+      // mode 2: h.out is free once the previous batch's bytes went back
+      if (mode == 2 && b >= (size_t)kHostSets && cudaStreamWaitEvent(ss, ev_out[k], 0) != cudaSuccess)
         return LZR_ERR_CUDA;
     } else if (cudaMemcpyAsync(h.in, (const uint8_t*)h_in + lo, len, cudaMemcpyHostToDevice, ss) != cudaSuccess) {
       return LZR_ERR_CUDA;
@@ -546,8 +566,10 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
       h_offsets[c0 + i] += running;
       tb += h_sizes[c0 + i];
     }
-    if (tb && cudaMemcpyAsync((uint8_t*)h_out + running, h.out, tb, cudaMemcpyDeviceToHost, ss) != cudaSuccess)
+    cudaStream_t ds = mode == 2 ? cin[1] : ss;
+    if (tb && cudaMemcpyAsync((uint8_t*)h_out + running, h.out, tb, cudaMemcpyDeviceToHost, ds) != cudaSuccess)
       return LZR_ERR_CUDA;
+    if (mode == 2 && cudaEventRecord(ev_out[b % kHostSets], ds) != cudaSuccess) return LZR_ERR_CUDA;
     running += tb;
     return LZR_OK;
   };
