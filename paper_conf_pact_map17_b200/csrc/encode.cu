@@ -434,6 +434,44 @@ __device__ __forceinline__ uint32_t walk_bound(uint32_t n, uint32_t k, uint32_t 
   return b < n ? b : n;
 }
 
+// (A/B on 1 x B200, 256 MiB, GB/s mix/text/zero-runs: fixed slope bounds
+// 51.8/28.2/81.5; A:B = 2:1 52.3/28.5/81.0; 1:1 52.2; 1:2 52.2; 3:1 52.4; 4:1 52.2;
+// 8:1 52.1.  LZR_WALK_CAND_A=0 restores walk_bound.)
+#ifndef LZR_WALK_CAND_A
+#define LZR_WALK_CAND_A 2u
+#endif
+#ifndef LZR_WALK_CAND_B
+#define LZR_WALK_CAND_B 1u
+#endif
+// Segment bounds from the candidate bitmap (LZR_WALK_CAND_A > 0): a word of 32
+// positions weighs A * (its candidate positions) + B (B ~ one literal-stretch
+// iteration); bounds are word starts splitting the total weight into K equal
+// parts.  Any bounds give the exact parse (meeting points), so this only moves
+// work between the walk segments.
+__device__ __forceinline__ uint32_t walk_bound_cand(const uint32_t* cand, uint32_t nwords,
+                                                    uint32_t n, uint32_t kk, uint32_t K,
+                                                    uint32_t tot, uint32_t lane) {
+  if (kk == 0) return 0;
+  if (kk >= K) return n;
+  const uint32_t t = (uint32_t)(((unsigned long long)tot * kk) / K);
+  uint32_t carry = 0;
+  for (uint32_t w0 = 0; w0 < nwords; w0 += 32) {
+    const uint32_t w = w0 + lane;
+    const uint32_t v = w < nwords ? LZR_WALK_CAND_A * __popc(cand[w]) + LZR_WALK_CAND_B : 0u;
+    uint32_t incl = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, incl, o);
+      if ((int)lane >= o) incl += y;
+    }
+    // first word whose exclusive cumulative weight reaches t
+    const uint32_t hit = __ballot_sync(kFull, w < nwords && carry + incl - v >= t);
+    if (hit) return min(n, (w0 + (uint32_t)(__ffs(hit) - 1)) << 5);
+    carry += __shfl_sync(kFull, incl, 31);
+  }
+  return n;
+}
+
 __device__ __forceinline__ uint32_t valid_mask(uint32_t n, uint32_t w) {
   const uint32_t base = w << 5;
   return n >= base + 32 ? 0xFFFFFFFFu : (n > base ? (1u << (n - base)) - 1u : 0u);
@@ -762,7 +800,24 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     {
       // later positions have more candidates: segment bounds balance a work
       // density growing ~linearly with the position (walk_bound)
-      const uint32_t start = walk_bound(n, k, K), nb = walk_bound(n, k + 1, K);
+      // up to 4 KiB (K <= 4): bounds from the candidate bitmap; above, the work
+      // per candidate grows along the chunk (longer lists), which the fixed
+      // slope models better (C = 8/16/32 KiB mix: 41.4/23.9/11.1 GB/s with the
+      // slope vs 41.1/23.5/10.8 with candidate weights)
+      uint32_t start, nb;
+      if (K <= 4 && LZR_WALK_CAND_A + 0 > 0) {
+        const uint32_t nwords = (n + 31) >> 5;
+        uint32_t tot = 0;
+        for (uint32_t w0 = 0; w0 < nwords; w0 += 32) {
+          const uint32_t w = w0 + lane;
+          tot += __reduce_add_sync(kFull, w < nwords ? LZR_WALK_CAND_A * __popc(S.cand[w]) + LZR_WALK_CAND_B : 0u);
+        }
+        start = walk_bound_cand(S.cand, nwords, n, k, K, tot, lane);
+        nb = walk_bound_cand(S.cand, nwords, n, k + 1, K, tot, lane);
+      } else {
+        start = walk_bound(n, k, K);
+        nb = walk_bound(n, k + 1, K);
+      }
       if (start < n && (k == 0 || start > 0))
         walk_segment<K, LZ>(S, d1, k, start, nb, n, P, nruns, a, lane);
     }
