@@ -416,13 +416,16 @@ HostSet carve(uint8_t* base, size_t batch, const lzr_params* p) {
 // batches' compressed bytes go back (D2H) and later batches' inputs come in
 // (H2D); a set is reused only after its D2H was issued on its own stream
 // (stream order).
+namespace {
 constexpr int kMaxHostSets = 8;
 // default 3 sets with shared copy streams (e2e sweep on 1 x B200, 256 MiB mix,
 // PCIe 55 GB/s one way / 93 both ways, tools/e2e_sweep.py; 8/16/32 MiB batches):
 // 3 sets 33.8/39.5/37.1 GB/s, 4 sets 37.6/38.6/36.4, 6 sets 35.6/36.0/32.6; a
 // copy stream per set 33.0/37.4/37.0 (3 sets); H2D on the compute stream
 // 32.6/37.0/36.5 (4 sets).  More sets split the link and the SMs over more
-// batches at once, so each batch's bytes arrive later
+// batches at once, so each batch's bytes arrive later.  With the cached
+// streams/events and launch attributes (no per-call / per-launch host setup):
+// 3 sets 12/16/24 MiB 40.0/43.6/43.0, 4 sets 44.0/44.0/42.0, 5 sets 43.6/43.0/41.5
 int host_sets() {  // LZR_HOST_SETS=2..8 overrides (tuning)
   static int v = -1;
   if (v < 0) {
@@ -443,6 +446,87 @@ int host_split() {
   }
   return v;
 }
+
+// Streams and events of the host pipeline.  Creating and destroying them on
+// every call costs host time that the pipeline's first batches wait for, so
+// each device keeps one cached set (created on first use, never destroyed;
+// state is only these handles).  A call that finds its device's set in use
+// (concurrent callers) creates a private set and destroys it afterwards.
+struct HostStreams {
+  cudaStream_t s[kMaxHostSets], cin[kMaxHostSets];
+  cudaEvent_t ev_in[kMaxHostSets], ev_kdone[kMaxHostSets], ev_out[kMaxHostSets];
+  int made = 0;       // sets created
+  bool cached = false;
+  bool busy = false;
+};
+constexpr int kMaxDevices = 64;
+std::mutex g_hs_mu;
+HostStreams g_hs[kMaxDevices];
+
+bool make_host_streams(HostStreams* h, int n) {
+  for (; h->made < n; ++h->made) {
+    const int i = h->made;
+    if (cudaStreamCreateWithFlags(&h->s[i], cudaStreamNonBlocking) != cudaSuccess) return false;
+    if (cudaStreamCreateWithFlags(&h->cin[i], cudaStreamNonBlocking) != cudaSuccess) {
+      cudaStreamDestroy(h->s[i]);
+      return false;
+    }
+    cudaEvent_t* evs[3] = {&h->ev_in[i], &h->ev_kdone[i], &h->ev_out[i]};
+    for (int e = 0; e < 3; ++e) {
+      if (cudaEventCreateWithFlags(evs[e], cudaEventDisableTiming) != cudaSuccess) {
+        for (int f = 0; f < e; ++f) cudaEventDestroy(*evs[f]);
+        cudaStreamDestroy(h->s[i]);
+        cudaStreamDestroy(h->cin[i]);
+        return false;
+      }
+    }
+  }
+  return true;
+}
+
+void destroy_host_streams(HostStreams* h) {
+  for (int i = 0; i < h->made; ++i) {
+    cudaStreamDestroy(h->s[i]);
+    cudaStreamDestroy(h->cin[i]);
+    cudaEventDestroy(h->ev_in[i]);
+    cudaEventDestroy(h->ev_kdone[i]);
+    cudaEventDestroy(h->ev_out[i]);
+  }
+  h->made = 0;
+}
+
+HostStreams* acquire_host_streams(int n) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+  if (dev >= 0 && dev < kMaxDevices) {
+    std::lock_guard<std::mutex> lk(g_hs_mu);
+    HostStreams* h = &g_hs[dev];
+    if (!h->busy) {
+      if (!make_host_streams(h, n)) return nullptr;  // partial sets stay cached
+      h->busy = true;
+      h->cached = true;
+      return h;
+    }
+  }
+  HostStreams* h = new HostStreams();
+  if (!make_host_streams(h, n)) {
+    destroy_host_streams(h);
+    delete h;
+    return nullptr;
+  }
+  return h;
+}
+
+void release_host_streams(HostStreams* h) {
+  if (h->cached) {
+    std::lock_guard<std::mutex> lk(g_hs_mu);
+    h->busy = false;
+    return;
+  }
+  destroy_host_streams(h);
+  delete h;
+}
+}  // namespace
 
 size_t lzr_compress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
   if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
@@ -469,53 +553,20 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
   const int kHostSets = host_sets();
   if (scratch_bytes < kHostSets * per) return LZR_ERR_CAPACITY;
   HostSet set[kMaxHostSets];
-  cudaStream_t s[kMaxHostSets], cin[kMaxHostSets];
-  cudaEvent_t ev_in[kMaxHostSets], ev_kdone[kMaxHostSets], ev_out[kMaxHostSets];
+  for (int i = 0; i < kHostSets; ++i) set[i] = carve((uint8_t*)d_scratch + i * per, batch_bytes, p);
   // split (mode >= 1): a set's H2D waits only for the kernels of the set's
   // previous batch (its input buffer), not for that batch's D2H of compressed
   // bytes (which reads the output buffer; mode 2: the kernels wait for that)
   const int mode = host_split();
   const bool split = mode >= 1;
-  int made = 0;
-  for (; made < kHostSets; ++made) {
-    set[made] = carve((uint8_t*)d_scratch + made * per, batch_bytes, p);
-    if (cudaStreamCreateWithFlags(&s[made], cudaStreamNonBlocking) != cudaSuccess) break;
-    if (cudaStreamCreateWithFlags(&cin[made], cudaStreamNonBlocking) != cudaSuccess) {
-      cudaStreamDestroy(s[made]);
-      break;
-    }
-    if (cudaEventCreateWithFlags(&ev_in[made], cudaEventDisableTiming) != cudaSuccess) {
-      cudaStreamDestroy(s[made]);
-      cudaStreamDestroy(cin[made]);
-      break;
-    }
-    if (cudaEventCreateWithFlags(&ev_kdone[made], cudaEventDisableTiming) != cudaSuccess) {
-      cudaStreamDestroy(s[made]);
-      cudaStreamDestroy(cin[made]);
-      cudaEventDestroy(ev_in[made]);
-      break;
-    }
-    if (cudaEventCreateWithFlags(&ev_out[made], cudaEventDisableTiming) != cudaSuccess) {
-      cudaStreamDestroy(s[made]);
-      cudaStreamDestroy(cin[made]);
-      cudaEventDestroy(ev_in[made]);
-      cudaEventDestroy(ev_kdone[made]);
-      break;
-    }
-  }
-  auto destroy = [&](int k) {
-    for (int i = 0; i < k; ++i) {
-      cudaStreamDestroy(s[i]);
-      cudaStreamDestroy(cin[i]);
-      cudaEventDestroy(ev_in[i]);
-      cudaEventDestroy(ev_kdone[i]);
-      cudaEventDestroy(ev_out[i]);
-    }
-  };
-  if (made < kHostSets) {
-    destroy(made);
-    return LZR_ERR_CUDA;
-  }
+  // streams and events: the device's cached pool when free, else a private set
+  HostStreams* hs = acquire_host_streams(kHostSets);
+  if (!hs) return LZR_ERR_CUDA;
+  cudaStream_t* s = hs->s;
+  cudaStream_t* cin = hs->cin;
+  cudaEvent_t* ev_in = hs->ev_in;
+  cudaEvent_t* ev_kdone = hs->ev_kdone;
+  cudaEvent_t* ev_out = hs->ev_out;
   const size_t nb = (n_bytes + batch_bytes - 1) / batch_bytes;
   const size_t chunks_per_batch = batch_bytes / C;
   uint64_t running = 0;
@@ -584,7 +635,7 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
     if ((cudaStreamSynchronize(s[i]) != cudaSuccess || cudaStreamSynchronize(cin[i]) != cudaSuccess) &&
         rc == LZR_OK)
       rc = LZR_ERR_CUDA;
-  destroy(kHostSets);
+  release_host_streams(hs);
   if (h_total) *h_total = running;
   t_launches = launches;
   return rc;

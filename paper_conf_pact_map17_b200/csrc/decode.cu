@@ -16,6 +16,8 @@
 // raw chunks are copied with 16-byte stores from funnel-shifted 4-byte loads.
 // Malformed streams set *err = min(1 + chunk index) (err pre-set to 0x7F7F7F7F,
 // fixed up to 0 afterwards when no chunk was corrupt).
+#include <mutex>
+
 #include "lzr_internal.cuh"
 
 namespace lzr {
@@ -201,9 +203,31 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   if (warps > kDecWarpsMax) warps = kDecWarpsMax;
   if (warps < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)warps * stride;
-  cudaError_t e = cudaFuncSetAttribute(lzr_decode_kernel,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // smem attribute + occupancy at this size, cached per device (host calls
+  // kept off the per-launch path)
+  static size_t c_smem[64] = {};
+  static int c_per_sm[64] = {};
+  static std::mutex mu;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
+  int per_sm = 0;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 0 && dev < 64 && c_smem[dev] == smem) per_sm = c_per_sm[dev];
+  }
+  if (per_sm == 0) {
+    e = cudaFuncSetAttribute(lzr_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    // as many CTAs as fit (shared memory bound), at most one wave of chunks
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel, warps * 32, smem);
+    if (e != cudaSuccess || per_sm < 1) per_sm = 1;
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 0 && dev < 64) {
+      c_smem[dev] = smem;
+      c_per_sm[dev] = per_sm;
+    }
+  }
   int32_t* errp = err;
   if (errp) {
     e = cudaMemsetAsync(errp, 0x7F, sizeof(int32_t), s);
@@ -214,10 +238,6 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
     e = cudaGetSymbolAddress((void**)&errp, g_scratch_err);
     if (e != cudaSuccess) return e;
   }
-  // as many CTAs as fit (shared memory bound), at most one wave of chunks
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel, warps * 32, smem);
-  if (e != cudaSuccess || per_sm < 1) per_sm = 1;
   size_t blocks = (N + warps - 1) / warps;
   const size_t cap = (size_t)sm_count * per_sm;
   if (blocks > cap) blocks = cap;

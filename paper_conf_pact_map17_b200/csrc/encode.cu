@@ -33,6 +33,8 @@
 //       in shared memory and written with 16-byte stores; raw fallback (R9).
 // The serial result is reproduced exactly: the best match at p depends only on
 // (chunk bytes, p, W, m, M), not on the parse.
+#include <mutex>
+
 #include "lzr_internal.cuh"
 
 namespace lzr {
@@ -985,16 +987,37 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   if (groups > 15) groups = 15;  // named barriers 1..15
   if (groups < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)groups * a.L.per_group;
-  cudaError_t err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // the smem attribute and the occupancy of this instantiation at this smem
+  // size, per device: host calls cached so that batch-by-batch callers (the
+  // host pipeline) do not pay them on every launch
+  struct Cached {
+    size_t smem;
+    int per_sm;
+  };
+  static Cached cache[64] = {};
+  static std::mutex mu;
+  int dev = 0;
+  cudaError_t err = cudaGetDevice(&dev);
   if (err != cudaSuccess) return err;
-  // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
-  int per_sm = 1;
-  if (MinBlocks<K, G1>::value > 1 &&
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1>,
-                                                    groups * 32 * K, smem) != cudaSuccess)
+  int per_sm = 0;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 0 && dev < 64 && cache[dev].smem == smem) per_sm = cache[dev].per_sm;
+  }
+  if (per_sm == 0) {
+    err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (err != cudaSuccess) return err;
+    // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
-  if (per_sm < 1) per_sm = 1;
+    if (MinBlocks<K, G1>::value > 1 &&
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1>,
+                                                      groups * 32 * K, smem) != cudaSuccess)
+      per_sm = 1;
+    if (per_sm < 1) per_sm = 1;
+    std::lock_guard<std::mutex> lk(mu);
+    if (dev >= 0 && dev < 64) cache[dev] = {smem, per_sm};
+  }
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
