@@ -337,3 +337,34 @@ def test_runs_structures_param_grid(lzr, ref, C, W, m):
     _check_full(lzr, ref, x, lzr.Params(chunk_size=C, window=W, min_match=m))
     z = synth.fill_host(C * 6, C, "zeroruns", seed=m)
     _check_full(lzr, ref, z, lzr.Params(chunk_size=C, window=W, min_match=m))
+
+
+def test_compress_host_concurrent_callers(lzr, ref):
+    """Three host threads in lzr_compress_host at once on one device: the first
+    takes the device's cached streams, the others private sets (capi.cu
+    HostStreams); every result equals the device path's, greedy and lazy."""
+    import threading
+
+    jobs = []
+    for t, (cls, parse) in enumerate([("mix", 0), ("text", 1), ("zeroruns", 0)]):
+        x = synth.fill_host((4 << 20) + 4096 * t + 77, 4096, cls, seed=40 + t)
+        jobs.append((x, lzr.Params(parse=parse)))
+    res = [None] * len(jobs)
+
+    def run(i):
+        x, p = jobs[i]
+        h = torch.from_numpy(x).pin_memory()
+        for _ in range(3):
+            res[i] = lzr.compress_host(h, p, batch_bytes=1 << 20)
+
+    ths = [threading.Thread(target=run, args=(i,)) for i in range(len(jobs))]
+    for th in ths:
+        th.start()
+    for th in ths:
+        th.join()
+    for (x, p), (h_out, h_sizes, h_offs, tot) in zip(jobs, res):
+        _, _, _, _, dtot, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, p)
+        assert tot == dtot
+        assert np.array_equal(h_sizes.numpy().view(np.uint32), g_sizes)
+        assert np.array_equal(h_offs.numpy().view(np.uint64), g_offs)
+        assert np.array_equal(h_out[:tot].numpy(), g_out)
