@@ -655,50 +655,98 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     //      round); split j's cursor of bucket h = start of h + counts of h in
     //      splits < j.  The other warps: zero the bitmaps, byte-change bitmap,
     //      walk state
-    const uint32_t kk = K == 1 ? 0 : k - 1, KK = K == 1 ? 1 : K - 1;  // helper warp index
-    if (k == 0) {
+#ifndef LZR_PAR_SCAN
+#define LZR_PAR_SCAN 1
+#endif
+    // K = 4 (C <= 4 KiB): the bucket scan is shared by the four warps -- each
+    // scans a quarter with a local carry, then adds the totals of the quarters
+    // before it -- instead of warp 0 alone while the others wait at the barrier
+    constexpr bool kParScan = LZR_PAR_SCAN && K == 4 && NS == 1;
+    if (kParScan && (B / 2) % (32 * K) == 0) {
+      const uint32_t q0 = k * (B / 2 / K), q1 = q0 + B / 2 / K;
       uint32_t carry = 0;
-      for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
-        const bool act = w0 + lane < B / 2;
-        const bool priv = skipr && w0 + lane < 128;  // buckets 2w, 2w+1 < 256: left empty
-        uint32_t c0 = 0, c1 = 0;  // totals of buckets 2w, 2w+1
-        for (uint32_t j = 0; j < NS; ++j) {
-          const uint32_t wv = act && !priv ? hist[j * (B / 2) + w0 + lane] : 0;
-          c0 += wv & 0xFFFFu;
-          c1 += wv >> 16;
-        }
-        const uint32_t sum = c0 + c1;
+      for (uint32_t w0 = q0; w0 < q1; w0 += 32) {
+        const uint32_t wi = w0 + lane;
+        const bool priv = skipr && wi < 128;  // buckets 2w, 2w+1 < 256: left empty
+        const uint32_t wv = priv ? 0u : hist[wi];
+        const uint32_t c0 = wv & 0xFFFFu, c1 = wv >> 16, sum = c0 + c1;
         uint32_t incl = sum;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
           const uint32_t t = __shfl_up_sync(kFull, incl, o);
           if ((int)lane >= o) incl += t;
         }
-        uint32_t e0 = incl - sum + carry, e1 = e0 + c0;  // running cursors
-        if (act) {
-          for (uint32_t j = 0; j < NS; ++j) {
-            const uint32_t wv = priv ? 0u : hist[j * (B / 2) + w0 + lane];
-            hist[j * (B / 2) + w0 + lane] = (e0 & 0xFFFFu) | (e1 << 16);
-            e0 += wv & 0xFFFFu;
-            e1 += wv >> 16;
-          }
-        }
+        const uint32_t e0 = incl - sum + carry, e1 = e0 + c0;
+        hist[wi] = (e0 & 0xFFFFu) | (e1 << 16);
         carry += __shfl_sync(kFull, incl, 31);
       }
-      if (lane == 0) S.ctrl[kCtrlIdx] = carry;  // index entries (P, or fewer when skipr)
-    }
-    if (K == 1 || k != 0) {
-      for (uint32_t i = kk * 32 + lane; i < nw; i += KK * 32) S.cand[i] = 0;
-      for (uint32_t i = kk * 32 + lane; i < K * a.L.tb_words; i += KK * 32) S.tb[i] = 0;
-      for (uint32_t w = kk; w < nw; w += KK) {  // change bitmap
+      if (lane == 0) S.ctrl[kCtrlProg + k] = carry;  // quarter total (prog is set up below)
+      for (uint32_t i = tid; i < nw; i += nthr) S.cand[i] = 0;
+      for (uint32_t i = tid; i < K * a.L.tb_words; i += nthr) S.tb[i] = 0;
+      for (uint32_t w = k; w < nw; w += K) {  // change bitmap
         const uint32_t i = (w << 5) + lane;
         const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
         const uint32_t b = __ballot_sync(kFull, ch);
         if (lane == 0) S.cb[w] = b;
       }
-      if (kk == 0 && lane < K) {
-        S.ctrl[kCtrlProg + lane] = 0;      // prog
-        S.ctrl[kCtrlProg + K + lane] = n;  // sync
+      GSYNC(14);
+      uint32_t base = 0, all = 0;
+      for (uint32_t j = 0; j < K; ++j) {
+        const uint32_t t = S.ctrl[kCtrlProg + j];
+        base += j < k ? t : 0u;
+        all += t;
+      }
+      if (base)
+        for (uint32_t wi = q0 + lane; wi < q1; wi += 32) hist[wi] += base | (base << 16);
+      if (k == 0 && lane == 0) S.ctrl[kCtrlIdx] = all;  // index entries
+      // (prog / sync are set up after the next barrier, once every warp has
+      // read the quarter totals: by the last warp, with the run ends)
+    } else {
+    const uint32_t kk = K == 1 ? 0 : k - 1, KK = K == 1 ? 1 : K - 1;  // helper warp index
+      if (k == 0) {
+        uint32_t carry = 0;
+        for (uint32_t w0 = 0; w0 < B / 2; w0 += 32) {
+          const bool act = w0 + lane < B / 2;
+          const bool priv = skipr && w0 + lane < 128;  // buckets 2w, 2w+1 < 256: left empty
+          uint32_t c0 = 0, c1 = 0;  // totals of buckets 2w, 2w+1
+          for (uint32_t j = 0; j < NS; ++j) {
+            const uint32_t wv = act && !priv ? hist[j * (B / 2) + w0 + lane] : 0;
+            c0 += wv & 0xFFFFu;
+            c1 += wv >> 16;
+          }
+          const uint32_t sum = c0 + c1;
+          uint32_t incl = sum;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(kFull, incl, o);
+            if ((int)lane >= o) incl += t;
+          }
+          uint32_t e0 = incl - sum + carry, e1 = e0 + c0;  // running cursors
+          if (act) {
+            for (uint32_t j = 0; j < NS; ++j) {
+              const uint32_t wv = priv ? 0u : hist[j * (B / 2) + w0 + lane];
+              hist[j * (B / 2) + w0 + lane] = (e0 & 0xFFFFu) | (e1 << 16);
+              e0 += wv & 0xFFFFu;
+              e1 += wv >> 16;
+            }
+          }
+          carry += __shfl_sync(kFull, incl, 31);
+        }
+        if (lane == 0) S.ctrl[kCtrlIdx] = carry;  // index entries (P, or fewer when skipr)
+      }
+      if (K == 1 || k != 0) {
+        for (uint32_t i = kk * 32 + lane; i < nw; i += KK * 32) S.cand[i] = 0;
+        for (uint32_t i = kk * 32 + lane; i < K * a.L.tb_words; i += KK * 32) S.tb[i] = 0;
+        for (uint32_t w = kk; w < nw; w += KK) {  // change bitmap
+          const uint32_t i = (w << 5) + lane;
+          const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
+          const uint32_t b = __ballot_sync(kFull, ch);
+          if (lane == 0) S.cb[w] = b;
+        }
+        if (kk == 0 && lane < K) {
+          S.ctrl[kCtrlProg + lane] = 0;      // prog
+          S.ctrl[kCtrlProg + K + lane] = n;  // sync
+        }
       }
     }
     GSYNC(3);
@@ -733,6 +781,10 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
       }
     }
     if (k == K - 1) {
+      if (kParScan && (B / 2) % (32 * K) == 0 && lane < K) {
+        S.ctrl[kCtrlProg + lane] = 0;      // prog
+        S.ctrl[kCtrlProg + K + lane] = n;  // sync
+      }
       for (uint32_t j = lane; j < min(nruns, a.L.max_runs); j += 32) {
         const uint32_t st = S.runs[j];
         S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
