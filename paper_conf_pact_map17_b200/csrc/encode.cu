@@ -681,14 +681,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         carry += __shfl_sync(kFull, incl, 31);
       }
       if (lane == 0) S.ctrl[kCtrlProg + k] = carry;  // quarter total (prog is set up below)
-      for (uint32_t i = tid; i < nw; i += nthr) S.cand[i] = 0;
-      for (uint32_t i = tid; i < K * a.L.tb_words; i += nthr) S.tb[i] = 0;
-      for (uint32_t w = k; w < nw; w += K) {  // change bitmap
-        const uint32_t i = (w << 5) + lane;
-        const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
-        const uint32_t b = __ballot_sync(kFull, ch);
-        if (lane == 0) S.cb[w] = b;
-      }
+      // (zeroing and the byte-change bitmap run during warp 0's scatter, below)
       GSYNC(14);
       uint32_t base = 0, all = 0;
       for (uint32_t j = 0; j < K; ++j) {
@@ -778,6 +771,23 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
           if (act && lane == 31u - __clz(peers[u])) cur[h[u]] = (uint16_t)(basev + __popc(peers[u]));
           __syncwarp();
         }
+      }
+    }
+    if (kParScan && (B / 2) % (32 * K) == 0 && k > 0) {
+      // while warp 0 scatters: warps 1 .. K-2 zero the bitmaps, the last warp
+      // builds the byte-change bitmap (its run ends below need it)
+      constexpr uint32_t kZ = K > 2 ? K - 2 : 1;  // zeroing warps (kParScan: K = 4)
+      if (k + 1 < K) {
+        for (uint32_t i = (k - 1) * 32 + lane; i < nw; i += kZ * 32) S.cand[i] = 0;
+        for (uint32_t i = (k - 1) * 32 + lane; i < K * a.L.tb_words; i += kZ * 32) S.tb[i] = 0;
+      } else {
+        for (uint32_t w = 0; w < nw; ++w) {
+          const uint32_t i = (w << 5) + lane;
+          const bool ch = (i == 0) || (i >= n) || (S.data[i] != S.data[i - 1]);
+          const uint32_t b = __ballot_sync(kFull, ch);
+          if (lane == 0) S.cb[w] = b;
+        }
+        __syncwarp();
       }
     }
     if (k == K - 1) {
