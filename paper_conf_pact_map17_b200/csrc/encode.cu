@@ -661,7 +661,9 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     // K = 4 (C <= 4 KiB): the bucket scan is shared by the four warps -- each
     // scans a quarter with a local carry, then adds the totals of the quarters
     // before it -- instead of warp 0 alone while the others wait at the barrier
-    constexpr bool kParScan = LZR_PAR_SCAN && K == 4 && NS == 1;
+    // (greedy only: in the lazy kernel the same change measured 38.5 -> 35.9
+    // GB/s mix -- a different register allocation of its longer walk)
+    constexpr bool kParScan = LZR_PAR_SCAN && K == 4 && NS == 1 && !LZ;
     if (kParScan && (B / 2) % (32 * K) == 0) {
       const uint32_t q0 = k * (B / 2 / K), q1 = q0 + B / 2 / K;
       uint32_t carry = 0;

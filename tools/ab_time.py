@@ -10,9 +10,10 @@ ap.add_argument("cls", nargs="*", default=["mix", "text", "zeroruns"])
 ap.add_argument("--mib", type=int, default=256)
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--chunk-size", type=int, default=4096)
+ap.add_argument("--parse", type=int, default=0)  # 1 = lazy (R21)
 a = ap.parse_args()
 n = a.mib << 20
-p = lzr.Params(chunk_size=a.chunk_size)
+p = lzr.Params(chunk_size=a.chunk_size, parse=a.parse)
 x = torch.empty(n, dtype=torch.uint8, device="cuda")
 ws = lzr.Workspace(n, p, x.device)
 res = []
