@@ -28,11 +28,12 @@ t = np.array(buf, dtype=np.float64).reshape(16, 4, 2)
 N = n // 4096
 tot = t.sum()
 print(f"class {a.cls}: cycles per chunk per warp (work / wait), K=4")
-for i, nm in enumerate(NAMES):
+for i, nm in list(enumerate(NAMES)) + [(14, "scan part 1")]:
     w = t[i, :, 0] / N
     z = t[i, :, 1] / N
     print(f"{i:2d} {nm:14s} " + "  ".join(f"w{k}:{w[k]:7.0f}/{z[k]:6.0f}" for k in range(4)))
-print("total work", t[:12, :, 0].sum() / N / 4, "wait", t[:12, :, 1].sum() / N / 4)
+ph = list(range(12)) + [14]
+print("total work", t[ph, :, 0].sum() / N / 4, "wait", t[ph, :, 1].sum() / N / 4)
 print("best_match: cycles/chunk/warp", [round(t[12, k, 0] / N) for k in range(4)],
       "calls/chunk/warp", [round(t[12, k, 1] / N, 1) for k in range(4)],
       "walk iterations/chunk/warp", [round(t[13, k, 1] / N, 1) for k in range(4)])
