@@ -699,6 +699,13 @@ def main():
             "gpu_over_cpu_e2e": round(e2e_v / cpu_v, 2) if e2e_v else None,
             "use_gpu_for_compression": bool((e2e_v or gpu_v) > cpu_v),
             "paper": "GPU 88.3% better than CPU (P:16 §3.2(3), other hardware; context)"}
+    # the paper's own CPU-vs-GPU compression figures with their hardware (context
+    # only: other hardware, no absolute B/s printed)
+    line["paper_context"] = {
+        "gpu": "AMD Radeon HD 7970", "cpu": "Intel (model garbled in the text)",
+        "gpu_compression": "~100K IOPS at low CR (P:18 §4(2)); ~0.41 GB/s at 4 KiB per I/O (derived)",
+        "cpu_compression": "~50K IOPS at low CR (P:18 §4(2)); ~0.20 GB/s (derived)",
+        "gpu_over_cpu": "1.883x (P:16 §3.2(3) '88.3% better')"}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if sharded:
