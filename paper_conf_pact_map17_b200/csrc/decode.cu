@@ -199,8 +199,20 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
     return cudaSuccess;
   }
   const uint32_t stride = align_up(C, 16);  // rebuilt chunk
+// Grid: 2 warps (chunks) per CTA and one CTA per 2 chunks, so the hardware
+// block scheduler balances chunks of very different cost (raw copies vs text)
+// as CTAs retire; a persistent one-wave grid of 16-warp CTAs left SMs idle at
+// the end (1 x B200, 256 MiB, output GB/s mix/text/zero-runs: 16-warp one-wave
+// 290/214/596; full grids of 16/8/4/2/1-warp CTAs 302/309/347/380/369 mix,
+// text 239-242 except 211 at 1 warp (32 CTAs per SM = 32 warps))
+#ifndef LZR_DEC_WARPS
+#define LZR_DEC_WARPS 2
+#endif
+#ifndef LZR_DEC_ONEWAVE
+#define LZR_DEC_ONEWAVE 0
+#endif
   int warps = smem_optin / (int)stride;
-  if (warps > kDecWarpsMax) warps = kDecWarpsMax;
+  if (warps > LZR_DEC_WARPS) warps = LZR_DEC_WARPS;
   if (warps < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)warps * stride;
   // smem attribute + occupancy at this size, cached per device (host calls
@@ -219,7 +231,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   if (per_sm == 0) {
     e = cudaFuncSetAttribute(lzr_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    // as many CTAs as fit (shared memory bound), at most one wave of chunks
+    // (LZR_DEC_ONEWAVE: at most one resident wave of CTAs, warps loop over chunks)
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel, warps * 32, smem);
     if (e != cudaSuccess || per_sm < 1) per_sm = 1;
     std::lock_guard<std::mutex> lk(mu);
@@ -240,7 +252,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   }
   size_t blocks = (N + warps - 1) / warps;
   const size_t cap = (size_t)sm_count * per_sm;
-  if (blocks > cap) blocks = cap;
+  if (LZR_DEC_ONEWAVE && blocks > cap) blocks = cap;
   lzr_decode_kernel<<<(unsigned)blocks, warps * 32, smem, s>>>(comp, sizes, offsets, n_bytes, C, m,
                                                               out, errp, N, stride);
   if (launches) ++*launches;
