@@ -216,8 +216,9 @@ def test_scan_sizes_large(lzr):
         assert int(tot.item()) == 12345 + int(s.sum(dtype=np.uint64))
 
 
-def test_compress_host_pipeline(lzr, ref):
-    n = (8 << 20) + 4096 * 3 + 100
+@pytest.mark.parametrize("n", [(8 << 20) + 4096 * 3 + 100, 8 << 20])
+def test_compress_host_pipeline(lzr, ref, n):
+    # (a ragged last chunk and an exact multiple of the batch size)
     x = synth.fill_host(n, 4096, "mix", seed=21)
     h = torch.from_numpy(x).pin_memory()
     for batch in [0, 1 << 20, 3 * 4096 * 128]:
