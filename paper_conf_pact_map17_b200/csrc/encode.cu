@@ -658,28 +658,41 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
 #ifndef LZR_PAR_SCAN
 #define LZR_PAR_SCAN 1
 #endif
+#ifndef LZR_PAR_SCAN8
+#define LZR_PAR_SCAN8 1
+#endif
     // K = 4 (C <= 4 KiB): the bucket scan is shared by the four warps -- each
     // scans a quarter with a local carry, then adds the totals of the quarters
     // before it -- instead of warp 0 alone while the others wait at the barrier
     // (greedy only: in the lazy kernel the same change measured 38.5 -> 35.9
     // GB/s mix -- a different register allocation of its longer walk)
-    constexpr bool kParScan = LZR_PAR_SCAN && K == 4 && NS == 1 && !LZ;
+    constexpr bool kParScan = LZR_PAR_SCAN && (K == 4 || (K == 8 && LZR_PAR_SCAN8)) && NS + 2 <= K && !LZ;
     if (kParScan && (B / 2) % (32 * K) == 0) {
       const uint32_t q0 = k * (B / 2 / K), q1 = q0 + B / 2 / K;
       uint32_t carry = 0;
       for (uint32_t w0 = q0; w0 < q1; w0 += 32) {
         const uint32_t wi = w0 + lane;
         const bool priv = skipr && wi < 128;  // buckets 2w, 2w+1 < 256: left empty
-        const uint32_t wv = priv ? 0u : hist[wi];
-        const uint32_t c0 = wv & 0xFFFFu, c1 = wv >> 16, sum = c0 + c1;
+        uint32_t c0 = 0, c1 = 0;  // totals of buckets 2w, 2w+1 over the splits
+        for (uint32_t j = 0; j < NS; ++j) {
+          const uint32_t wv = priv ? 0u : hist[j * (B / 2) + wi];
+          c0 += wv & 0xFFFFu;
+          c1 += wv >> 16;
+        }
+        const uint32_t sum = c0 + c1;
         uint32_t incl = sum;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
           const uint32_t t = __shfl_up_sync(kFull, incl, o);
           if ((int)lane >= o) incl += t;
         }
-        const uint32_t e0 = incl - sum + carry, e1 = e0 + c0;
-        hist[wi] = (e0 & 0xFFFFu) | (e1 << 16);
+        uint32_t e0 = incl - sum + carry, e1 = e0 + c0;  // split j's cursors: + splits < j
+        for (uint32_t j = 0; j < NS; ++j) {
+          const uint32_t wv = priv ? 0u : hist[j * (B / 2) + wi];
+          hist[j * (B / 2) + wi] = (e0 & 0xFFFFu) | (e1 << 16);
+          e0 += wv & 0xFFFFu;
+          e1 += wv >> 16;
+        }
         carry += __shfl_sync(kFull, incl, 31);
       }
       if (lane == 0) S.ctrl[kCtrlProg + k] = carry;  // quarter total (prog is set up below)
@@ -692,7 +705,8 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         all += t;
       }
       if (base)
-        for (uint32_t wi = q0 + lane; wi < q1; wi += 32) hist[wi] += base | (base << 16);
+        for (uint32_t j = 0; j < NS; ++j)
+          for (uint32_t wi = q0 + lane; wi < q1; wi += 32) hist[j * (B / 2) + wi] += base | (base << 16);
       if (k == 0 && lane == 0) S.ctrl[kCtrlIdx] = all;  // index entries
       // (prog / sync are set up after the next barrier, once every warp has
       // read the quarter totals: by the last warp, with the run ends)
@@ -775,13 +789,13 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         }
       }
     }
-    if (kParScan && (B / 2) % (32 * K) == 0 && k > 0) {
-      // while warp 0 scatters: warps 1 .. K-2 zero the bitmaps, the last warp
-      // builds the byte-change bitmap (its run ends below need it)
-      constexpr uint32_t kZ = K > 2 ? K - 2 : 1;  // zeroing warps (kParScan: K = 4)
+    if (kParScan && (B / 2) % (32 * K) == 0 && k >= NS) {
+      // while warps < NS scatter: warps NS .. K-2 zero the bitmaps, the last
+      // warp builds the byte-change bitmap (its run ends below need it)
+      constexpr uint32_t kZ = K > NS + 1 ? K - 1 - NS : 1;  // zeroing warps
       if (k + 1 < K) {
-        for (uint32_t i = (k - 1) * 32 + lane; i < nw; i += kZ * 32) S.cand[i] = 0;
-        for (uint32_t i = (k - 1) * 32 + lane; i < K * a.L.tb_words; i += kZ * 32) S.tb[i] = 0;
+        for (uint32_t i = (k - NS) * 32 + lane; i < nw; i += kZ * 32) S.cand[i] = 0;
+        for (uint32_t i = (k - NS) * 32 + lane; i < K * a.L.tb_words; i += kZ * 32) S.tb[i] = 0;
       } else {
         for (uint32_t w = 0; w < nw; ++w) {
           const uint32_t i = (w << 5) + lane;
