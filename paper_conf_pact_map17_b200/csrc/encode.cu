@@ -661,6 +661,12 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
 #ifndef LZR_PAR_SCAN8
 #define LZR_PAR_SCAN8 1
 #endif
+// blocks of 32 positions per scatter round (their MATCH.ANY latencies
+// overlap): 8 at K = 4 (mix/text/zero-runs 53.1/28.8/83.5 -> 53.9/29.2/80.3;
+// 2 blocks: 52.1), 4 at K = 8 (8 KiB mix 42.6 vs 42.0 with 8)
+#ifndef LZR_SCATTER_BLOCKS
+#define LZR_SCATTER_BLOCKS (K == 4 ? 8 : 4)
+#endif
     // K = 4 (C <= 4 KiB): the bucket scan is shared by the four warps -- each
     // scans a quarter with a local carry, then adds the totals of the quarters
     // before it -- instead of warp 0 alone while the others wait at the barrier
@@ -768,18 +774,18 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     if (k < NS) {
       uint16_t* cur = S.slot + k * B;
       const uint32_t pe = min(P, (k + 1) * SS);
-      for (uint32_t p0 = k * SS; p0 < pe; p0 += 128) {
-        uint32_t h[4], peers[4];
+      for (uint32_t p0 = k * SS; p0 < pe; p0 += 32 * LZR_SCATTER_BLOCKS) {
+        uint32_t h[LZR_SCATTER_BLOCKS], peers[LZR_SCATTER_BLOCKS];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < LZR_SCATTER_BLOCKS; ++u) {
           const uint32_t p = p0 + 32 * u + lane;
           h[u] = p < pe ? khash(ld32u(S.data, p) & a.kmask, hb, a.kmask) : 0xFFFFFFFFu;
           if (skipr && h[u] < 256u) h[u] = 0xFFFFFFFFu;  // not indexed
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) peers[u] = __match_any_sync(kFull, h[u]);
+        for (int u = 0; u < LZR_SCATTER_BLOCKS; ++u) peers[u] = __match_any_sync(kFull, h[u]);
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < LZR_SCATTER_BLOCKS; ++u) {
           const bool act = h[u] != 0xFFFFFFFFu;
           const uint32_t basev = act ? cur[h[u]] : 0;
           if (act) S.sorted[basev + __popc(peers[u] & lt)] = (uint16_t)(p0 + 32 * u + lane);
