@@ -663,9 +663,10 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
 #endif
 // blocks of 32 positions per scatter round (their MATCH.ANY latencies
 // overlap): 8 at K = 4 (mix/text/zero-runs 53.1/28.8/83.5 -> 53.9/29.2/80.3;
-// 2 blocks: 52.1), 4 at K = 8 (8 KiB mix 42.6 vs 42.0 with 8)
+// 2 blocks: 52.1), 4 at K = 8 (8 KiB mix 42.6 vs 42.0 with 8) and in the lazy
+// kernel (38.4 vs 37.2 with 8)
 #ifndef LZR_SCATTER_BLOCKS
-#define LZR_SCATTER_BLOCKS (K == 4 ? 8 : 4)
+#define LZR_SCATTER_BLOCKS (K == 4 && !LZ ? 8 : 4)
 #endif
     // K = 4 (C <= 4 KiB): the bucket scan is shared by the four warps -- each
     // scans a quarter with a local carry, then adds the totals of the quarters
