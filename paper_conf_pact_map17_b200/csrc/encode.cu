@@ -308,6 +308,9 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 // at q + 1 is not strictly longer; otherwise q is a literal and the walk moves
 // to q + 1, whose best match is then already known (cached).  The decision at
 // q depends on q alone, so the meeting-point argument above is unchanged.
+#ifndef LZR_PUB
+#define LZR_PUB 64  // progress published every LZR_PUB bytes of parse
+#endif
 template <int K, bool LZ>
 __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
                                              uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
@@ -404,7 +407,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     }
     p = bits ? q + tok_len : q;
     // publish progress (a later publish only delays meeting; warp 0's is never read)
-    if (k > 0 && (p - pub >= 64 || p >= n)) {
+    if (k > 0 && (p - pub >= LZR_PUB || p >= n)) {
       pub = p;
       if (lane == 0) {
         fence_acq_rel_cta();  // recorded token bits before the progress word
