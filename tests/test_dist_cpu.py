@@ -36,7 +36,7 @@ class OracleOps:
         import oracle
 
         self.ref = oracle
-        self.rp = oracle.Params(chunk_size=p.chunk_size)
+        self.rp = oracle.Params(chunk_size=p.chunk_size, parse=p.parse)
 
     def compress(self, x):
         out, sizes, offs, total = self.ref.compress(x.numpy(), self.rp, n_threads=1)
@@ -65,7 +65,7 @@ def _free_port():
     return port
 
 
-def _worker(rank, world, port, n_global, C, q):
+def _worker(rank, world, port, n_global, C, q, parse=0):
     import synth
     import paper_conf_pact_map17_b200 as lzr
 
@@ -73,7 +73,7 @@ def _worker(rank, world, port, n_global, C, q):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        p = lzr.Params(chunk_size=C)
+        p = lzr.Params(chunk_size=C, parse=parse)
         sc = ShardedCompressor(n_global, p, None, "cpu", ops=OracleOps(p))
         x_local = synth.fill_host(sc.n_local, C, "mix", seed=77, first_chunk=sc.lo) if sc.n_local else np.zeros(0, np.uint8)
         res = sc(torch.from_numpy(np.ascontiguousarray(x_local)))
@@ -85,8 +85,9 @@ def _worker(rank, world, port, n_global, C, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,nchunks,tail", [(2, 37, 100), (3, 10, 0), (4, 3, 17), (2, 1, 5)])
-def test_sharded_offsets_match_single_process(ref, world, nchunks, tail):
+@pytest.mark.parametrize("world,nchunks,tail,parse", [(2, 37, 100, 0), (3, 10, 0, 0), (4, 3, 17, 0), (2, 1, 5, 0),
+                                                     (2, 37, 100, 1)])
+def test_sharded_offsets_match_single_process(ref, world, nchunks, tail, parse):
     import synth
 
     C = 512
@@ -94,7 +95,7 @@ def test_sharded_offsets_match_single_process(ref, world, nchunks, tail):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, n_global, C, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, n_global, C, q, parse)) for r in range(world)]
     for pr in procs:
         pr.start()
     results = [q.get(timeout=120) for _ in range(world)]
@@ -102,7 +103,7 @@ def test_sharded_offsets_match_single_process(ref, world, nchunks, tail):
         pr.join(timeout=60)
         assert pr.exitcode == 0
     x = synth.fill_host(n_global, C, "mix", seed=77)
-    r_out, r_sizes, r_offs, r_tot = ref.compress(x, ref.Params(chunk_size=C))
+    r_out, r_sizes, r_offs, r_tot = ref.compress(x, ref.Params(chunk_size=C, parse=parse))
     N = ref.num_chunks(n_global, ref.Params(chunk_size=C))
     for rank, lo, hi, goffs, gtot, out_local, sizes_all in sorted(results, key=lambda t: t[0]):
         assert gtot == r_tot
