@@ -514,7 +514,10 @@ template <int K, bool G1 = false>
 struct MinBlocks {
   static constexpr int value = G1 ? (K == 4 ? 9 : 1) : (K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1));
 };
-constexpr uint32_t kG1MaxWaves = 12;  // launches of fewer chunk waves than this use G1
+#ifndef LZR_G1_MAX_WAVES
+#define LZR_G1_MAX_WAVES 12u
+#endif
+constexpr uint32_t kG1MaxWaves = LZR_G1_MAX_WAVES;  // launches of fewer chunk waves than this use G1
 
 template <int K, int NS, bool LZ, bool G1>
 __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::value)
