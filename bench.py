@@ -12,8 +12,12 @@ before timing (synthetic, seeded; DESIGN.md §Input recipe) and are larger than
 L2 (256 MiB per GPU vs 126 MB), so L2 is not flushed between steps.
 
 N = 1: config 2 of BASELINE.json (256 MiB mixed-compressibility stream).
-N > 1 (torchrun, one rank per GPU): weak scaling, 256 MiB per rank of one
-global mixed stream, sharded by contiguous chunk ranges.
+N > 1 (one rank per GPU): weak scaling, 256 MiB per rank of one global mixed
+stream, sharded by contiguous chunk ranges.  Started under torchrun (the
+driver's launch) or, when `--gpus N` is given without it, re-launched by this
+script through torch.distributed.run with N ranks.  `--backend gloo` runs the
+exchange over gloo with host-staged tensors, which lets N ranks share fewer
+GPUs (a functional run of the sharded path on one GPU, not a scaling number).
 
 --impl reference times the CPU oracle (oracle/, plain serial greedy LZ77,
 thread-per-chunk on the host cores) on a bounded sample of the same workload.
@@ -60,7 +64,96 @@ def parse():
                     help="W < C (SURVEY.md §8(f) N4); default W = C (the configs)")
     ap.add_argument("--parse", default="greedy", choices=["greedy", "lazy"],
                     help="parse rule (DESIGN.md R8 greedy, R21 one-step lazy; SURVEY.md §8(f) N4)")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N > 1 (gloo: host-staged exchange; ranks may "
+                         "share a GPU)")
+    ap.add_argument("--no-per-class", action="store_true")
+    ap.add_argument("--cpu-max-seconds", type=float, default=120.0,
+                    help="time cap of the oracle run (cpu_baseline); configs 1 and 2 run it over "
+                         "the whole stream unless the cap is hit")
     return ap.parse_args()
+
+
+def _free_port() -> int:
+    import socket
+
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def relaunch(a) -> int:
+    """`--gpus N` (N > 1) outside torchrun: start N ranks of this script through
+    torch.distributed.run on this node (the driver's own launch line)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={_free_port()}",
+           os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
+class Ranks:
+    """This process's place in the job: one rank per GPU (LOCAL_RANK), a
+    process group when started under torchrun, and the cross-rank reductions
+    of the timing (on the device for NCCL, on the host for gloo)."""
+
+    def __init__(self, a):
+        import torch
+        import torch.distributed as dist
+
+        self.dist = dist
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        self.sharded = "WORLD_SIZE" in os.environ and "MASTER_ADDR" in os.environ
+        if self.world != a.gpus:
+            raise SystemExit(f"bench.py: --gpus {a.gpus} but WORLD_SIZE={self.world}")
+        ndev = torch.cuda.device_count()
+        if ndev == 0:
+            raise SystemExit("bench.py needs a CUDA device (there is no CPU path)")
+        self.backend = a.backend if self.sharded else None
+        if self.local >= ndev and a.backend == "nccl":
+            raise SystemExit(f"bench.py: rank {self.local} but {ndev} GPU(s); NCCL needs one GPU per "
+                             "rank (--backend gloo lets ranks share a GPU)")
+        self.dev = torch.device("cuda", self.local % ndev)
+        self.share_gpu = self.world > ndev
+        torch.cuda.set_device(self.dev)
+        if self.sharded:
+            kw = {"device_id": self.dev} if a.backend == "nccl" else {}
+            dist.init_process_group(a.backend, **kw)
+
+    def _tensor(self, vals):
+        import torch
+
+        dev = self.dev if self.backend == "nccl" else "cpu"
+        return torch.tensor(vals, dtype=torch.float64, device=dev)
+
+    def reduce(self, x: float, op: str = "max") -> float:
+        if not self.sharded:
+            return x
+        t = self._tensor([x])
+        self.dist.all_reduce(t, op={"max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM}[op])
+        return float(t.item())
+
+    def gather(self, vals) -> list:
+        """[world][len(vals)] of every rank's values."""
+        if not self.sharded:
+            return [list(vals)]
+        import torch
+
+        t = self._tensor(list(vals))
+        out = [torch.empty_like(t) for _ in range(self.world)]
+        self.dist.all_gather(out, t)
+        return [o.cpu().tolist() for o in out]
+
+    def barrier(self):
+        if self.sharded:
+            self.dist.barrier()
+
+    def close(self):
+        if self.sharded:
+            self.dist.destroy_process_group()
 
 
 def peaks():
@@ -136,18 +229,19 @@ class ClockSampler:
 
 
 def _profile_entry(workload: str):
+    """The committed ncu summary of this workload, only if it was captured on
+    the kernel sources this run is built from (build hash, _build.source_hash)."""
+    from paper_conf_pact_map17_b200._build import source_hash
+
     path = os.path.join(ROOT, "profiles", "encode_ncu_summary.json")
     try:
         with open(path) as f:
-            return json.load(f).get(workload)
+            e = json.load(f).get(workload)
     except Exception:
         return None
-
-
-def traffic_from_profiles(workload: str):
-    """dram read+write bytes per encode launch from the committed ncu summary."""
-    e = _profile_entry(workload)
-    return float(e["dram_bytes_per_launch"]) if e else None
+    if not e or e.get("build") != source_hash():
+        return None
+    return e
 
 
 def issue_limiter(workload: str, enc_avg_s: float, sm_mhz, n_sms: int):
@@ -167,28 +261,40 @@ def issue_limiter(workload: str, enc_avg_s: float, sm_mhz, n_sms: int):
             "warp_inst_per_launch": inst, "source": e.get("source")}
 
 
-def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, sample_bytes):
-    """Oracle (thread-per-chunk on all host cores) on the first chunks of the same
-    stream; also checks those chunks against the GPU output byte for byte."""
+def cpu_baseline(x_host, p_gpu, g_sizes, g_offs, g_out, max_seconds, limit_chunks=None,
+                 batch_bytes=16 << 20):
+    """The oracle (thread-per-chunk on all host cores, §3.2(1)) over the
+    timed stream in 16 MiB batches -- the whole stream unless `limit_chunks` or
+    the time cap stops it -- with every batch's sizes, offsets and bytes
+    compared to the GPU output of the same chunks."""
     import numpy as np
 
     import oracle
 
     C = p_gpu.chunk_size
-    nchunks = max(1, min(len(g_sizes), sample_bytes // C))
-    xs = x_host[: nchunks * C]
+    N = len(g_sizes) if limit_chunks is None else min(len(g_sizes), limit_chunks)
     cores = len(os.sched_getaffinity(0))
-    t0 = time.perf_counter()
-    r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, oracle.Params(chunk_size=C, window=p_gpu.window,
-                                                                  parse=p_gpu.parse),
-                                                   n_threads=cores)
-    dt = time.perf_counter() - t0
-    ok = bool(np.array_equal(r_sizes, g_sizes[:nchunks]) and np.array_equal(r_offs, g_offs[:nchunks])
-              and np.array_equal(r_out, g_out[: int(r_tot)]))
-    return {"value": round(xs.size / dt / 1e9, 6), "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": f"first {nchunks} chunks ({xs.size / 2**20:.0f} MiB) of the timed stream, "
-                      f"thread-per-chunk, {dt:.1f} s",
-            "parity_vs_gpu": "bit-exact" if ok else "MISMATCH"}
+    rp = oracle.Params(chunk_size=C, window=p_gpu.window, parse=p_gpu.parse)
+    per = max(1, batch_bytes // C)
+    done, dt, ok = 0, 0.0, True
+    while done < N and dt < max_seconds:
+        hi = min(N, done + per)
+        xs = x_host[done * C: min(x_host.size, hi * C)]
+        t0 = time.perf_counter()
+        r_out, r_sizes, r_offs, r_tot = oracle.compress(xs, rp, n_threads=cores)
+        dt += time.perf_counter() - t0
+        base = int(g_offs[done])
+        ok = ok and bool(np.array_equal(r_sizes, g_sizes[done:hi])
+                         and np.array_equal(r_offs + np.uint64(base), g_offs[done:hi])
+                         and np.array_equal(r_out, g_out[base: base + int(r_tot)]))
+        done = hi
+    nbytes = min(x_host.size, done * C)
+    what = (f"all {done} chunks ({nbytes / 2**20:.0f} MiB) of the timed stream" if done == len(g_sizes)
+            else f"first {done} of {len(g_sizes)} chunks ({nbytes / 2**20:.0f} MiB) of the timed stream"
+            + (" (time cap)" if dt >= max_seconds else ""))
+    return {"value": round(nbytes / dt / 1e9, 6), "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{what}, thread-per-chunk, 16 MiB batches, {dt:.1f} s",
+            "parity_vs_gpu": ("bit-exact" if ok else "MISMATCH") + f" ({done} chunks)"}
 
 
 PARSES = {"greedy": 0, "lazy": 1}  # lzr_params.parse (include/lzr.h)
@@ -276,20 +382,13 @@ def run_dedup(a):
     logical_value = logical stream bytes per second."""
     import numpy as np
     import torch
-    import torch.distributed as dist
 
     import synth
     import paper_conf_pact_map17_b200 as lzr
-    from paper_conf_pact_map17_b200.dist import ShardedDedup, shard_range
+    from paper_conf_pact_map17_b200.dist import ShardedDedup, all_gather_into, shard_range
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    grank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    dev = torch.device("cuda", local)
-    torch.cuda.set_device(dev)
-    sharded = "WORLD_SIZE" in os.environ and "MASTER_ADDR" in os.environ
-    if sharded:
-        dist.init_process_group("nccl", device_id=dev)
+    R = Ranks(a)
+    world, grank, dev, sharded = R.world, R.rank, R.dev, R.sharded
     C = a.chunk_size
     p = lzr.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse])
     n_glob = ((a.bytes_per_rank * world if a.bytes_per_rank else (16 << 30)) // C) * C
@@ -354,35 +453,27 @@ def run_dedup(a):
         lzr.compress_compact(ubuf[:nub], p, ws)
         launches[0] += lzr.last_launch_count()
         if sharded:  # per-rank compressed totals -> global layout (8 B per rank)
-            dist.all_gather_into_tensor(totals_all, ws.total)
+            all_gather_into(totals_all, ws.total)
 
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
-    if sharded:
-        dist.barrier()
+    R.barrier()
     launches[0] = 0
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev.index) as clk:
         torch.cuda.synchronize()
-        if sharded:
-            dist.barrier()
+        R.barrier()
         t0.record(stream)
         for _ in range(a.steps):
             step(record=True)
         t1.record(stream)
         torch.cuda.synchronize()
-        if sharded:
-            dist.barrier()
-    ms = t0.elapsed_time(t1)
-    nub_all = nub
-    if sharded:
-        tt = torch.tensor([ms, float(nub)], dtype=torch.float64, device=dev)
-        mx = tt[:1].clone()
-        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
-        sm = tt[1:].clone()
-        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
-        ms, nub_all = float(mx.item()), int(sm.item())
+        R.barrier()
+    ms_rank = t0.elapsed_time(t1)
+    per_rank_ms = [r[0] / a.steps for r in R.gather([ms_rank])]
+    ms = R.reduce(ms_rank, "max")
+    nub_all = int(R.reduce(float(nub), "sum"))
     ms_step = ms / a.steps
     enc_ms = [e0.elapsed_time(e1) for e0, e1 in zip(ev["e0"], ev["e1"])]
     dedup_ms = [d.elapsed_time(e0) for d, e0 in zip(ev["d"], ev["e0"])]
@@ -404,26 +495,29 @@ def run_dedup(a):
         "config": {"workload": workload, "global_bytes": n_glob, "unique_bytes": nub_all,
                    "dedup_ratio": round(n_glob / max(1, nub_all), 4), "chunk_size": C, "window": a.window or C,
                    "min_match": 4, "max_match": 259, "parse": a.parse,
-                   "parallelism": (f"dp{world}: contiguous chunk shards; global index by NCCL "
-                                   "all-to-all to fingerprint owners; all-gather of totals")
+                   "parallelism": (f"dp{world}: contiguous chunk shards; global index by {R.backend} "
+                                   "all-to-all to fingerprint owners; all-gather of totals"
+                                   + (" (ranks share a GPU: functional run)" if R.share_gpu else ""))
                    if sharded else "1 GPU",
                    "l2": "inputs larger than L2 (126 MB); no flush",
                    "compression_ratio": round(nub / max(1, total), 4),
                    "raw_chunk_fraction": round(float(raw.mean()), 4)},
         "logical_value": round(n_glob / (ms_step / 1e3) / 1e9, 4),
+        "per_rank_ms": [round(v, 4) for v in per_rank_ms],
+        "rank_spread": round((max(per_rank_ms) - min(per_rank_ms)) / max(per_rank_ms), 4),
         "dedup": {"ms_per_step": round(statistics.mean(dedup_ms), 4),
                   "logical_GBps": round(n_glob / (statistics.mean(dedup_ms) / 1e3) / 1e9, 3),
                   "what": "index reset + SHA-1 fingerprints + insert/lookup + unique scan + gather"},
         "roofline": {"bound": "hbm", "kernel": "lzr_encode_kernel", "achieved": round(achieved, 3),
                      "peak": hbm_peak, "unit": "GB/s", "frac": round(achieved / hbm_peak, 6),
-                     "traffic": traffic_from_profiles(workload), "peak_source": peak_src,
+                     "traffic": None, "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": enc_algo_bytes,
                      "avg_launch_ms": round(enc_avg_s * 1e3, 4),
                      "share_of_step": round(statistics.mean(enc_ms) / ms_step, 4)},
         "clocks": clk.summary(),
         "gpu_launches": launches[0],
     }
-    if grank == 0 and not a.no_cpu:
+    if world == 1 and not a.no_cpu:
         import oracle
 
         smp = min(n, (a.cpu_sample_bytes // C) * C)
@@ -444,12 +538,47 @@ def run_dedup(a):
                                 "index_parity_vs_gpu": "bit-exact" if ok else "MISMATCH"}
     if grank == 0:
         print(json.dumps(line), flush=True)
-    if sharded:
-        dist.destroy_process_group()
+    R.close()
+
+
+def per_class(lzr, synth, p, n, dev, stream, steps=5, warmup=2):
+    """GPU GB/s and compression ratio per class
+    (text / random / zero-runs) on their own 256 MiB streams, compress
+    (encode + scan/compaction) and decompress, device-resident, CUDA events."""
+    import torch
+
+    x = torch.empty(n, dtype=torch.uint8, device=dev)
+    ws = lzr.Workspace(n, p, dev)
+    y = torch.empty(n, dtype=torch.uint8, device=dev)
+    err = torch.zeros(1, dtype=torch.int32, device=dev)
+    res = {}
+    for cls in ("text", "random", "zeroruns"):
+        synth.fill_device(x, p.chunk_size, cls)
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        for _ in range(warmup):
+            lzr.compress(x, p, ws=ws)
+        e[0].record(stream)
+        for _ in range(steps):
+            lzr.compress(x, p, ws=ws)
+        e[1].record(stream)
+        for _ in range(steps):
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n, p, y, err)
+        e[2].record(stream)
+        torch.cuda.synchronize()
+        tot = int(ws.total.item())
+        ok = int(err.item()) == 0 and bool(torch.equal(y, x))
+        res[cls] = {"compress_gbs": round(n * steps / (e[0].elapsed_time(e[1]) / 1e3) / 1e9, 3),
+                    "compression_ratio": round(n / max(1, tot), 4),
+                    "decompress_gbs": round(n * steps / (e[1].elapsed_time(e[2]) / 1e3) / 1e9, 3),
+                    "round_trip": "ok" if ok else "MISMATCH"}
+    del x, ws, y
+    return res
 
 
 def main():
     a = parse()
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch(a))
     if a.impl == "reference":
         run_reference(a)
         return
@@ -458,21 +587,13 @@ def main():
         return
     import numpy as np
     import torch
-    import torch.distributed as dist
 
     import synth
     import paper_conf_pact_map17_b200 as lzr
     from paper_conf_pact_map17_b200.dist import ShardedCompressor
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    # under torchrun the sharded path (NCCL all-gather of sizes) runs even at N = 1
-    sharded = "WORLD_SIZE" in os.environ and "MASTER_ADDR" in os.environ
-    if sharded:
-        dist.init_process_group("nccl", device_id=dev)
+    R = Ranks(a)
+    world, rank, dev, sharded = R.world, R.rank, R.dev, R.sharded
     C = a.chunk_size
     p = lzr.Params(chunk_size=C, window=a.window, parse=PARSES[a.parse])
     # workload (BASELINE.json configs); weak = fixed bytes per GPU, strong = fixed total
@@ -493,71 +614,58 @@ def main():
         sc = ShardedCompressor(n_glob, p, None, dev)
         n_rank = sc.n_local
         first = sc.lo
+        ws = sc.ops.ws
     else:
         n_rank = n_glob
         first = 0
+        ws = lzr.Workspace(n_rank, p, dev)
     x = torch.empty(n_rank, dtype=torch.uint8, device=dev)
     synth.fill_device(x, C, a.cls, first_chunk=first)
-    ws = lzr.Workspace(n_rank, p, dev)
-    if sharded:
-        sc.ops.ws = ws
-        sc.ops.bind_sizes(sc.sizes_pad)
 
     launches = [0]
 
     def step(ev_enc=None):
-        if sharded:
-            if ev_enc is not None:
-                ev_enc[0].record(stream)
-            lzr.compress_encode(x, p, ws)
-            launches[0] += lzr.last_launch_count()
-            if ev_enc is not None:
-                ev_enc[1].record(stream)
-            lzr.compress_compact(x, p, ws)
-            launches[0] += lzr.last_launch_count()
-            dist.all_gather_into_tensor(sc.sizes_all, sc.sizes_pad)
+        if ev_enc is not None:
+            ev_enc[0].record(stream)
+        lzr.compress_encode(x, p, ws)
+        launches[0] += lzr.last_launch_count()
+        if ev_enc is not None:
+            ev_enc[1].record(stream)
+        lzr.compress_compact(x, p, ws)
+        launches[0] += lzr.last_launch_count()
+        if sharded:  # sizes -> every rank, global offsets by the device scan
+            sc.ops.all_gather(sc.sizes_all, sc.sizes_pad, None)
             lzr.scan_sizes(sc.sizes_all, 0, offsets=sc.offsets_all, total=sc.global_total)
-            launches[0] += lzr.last_launch_count()
-        else:
-            if ev_enc is not None:
-                ev_enc[0].record(stream)
-            lzr.compress_encode(x, p, ws)
-            launches[0] += lzr.last_launch_count()
-            if ev_enc is not None:
-                ev_enc[1].record(stream)
-            lzr.compress_compact(x, p, ws)
             launches[0] += lzr.last_launch_count()
 
     for _ in range(a.warmup):
         step()
     torch.cuda.synchronize()
-    if sharded:
-        dist.barrier()
-    enc_events = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                  for _ in range(a.steps)]
+    R.barrier()
+    mk = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    enc_events = [(mk(), mk()) for _ in range(a.steps)]
+    step_ev = [mk() for _ in range(a.steps + 1)]
     launches[0] = 0
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev.index) as clk:
         torch.cuda.synchronize()
-        if sharded:
-            dist.barrier()
-        t_start.record(stream)
+        R.barrier()
+        step_ev[0].record(stream)
         for k in range(a.steps):
             step(enc_events[k])
-        t_end.record(stream)
+            step_ev[k + 1].record(stream)
         torch.cuda.synchronize()
-        if sharded:
-            dist.barrier()
-    ms = t_start.elapsed_time(t_end)
+        R.barrier()
+    step_ms = [step_ev[k].elapsed_time(step_ev[k + 1]) for k in range(a.steps)]
+    ms_rank = sum(step_ms)
     enc_ms = [e0.elapsed_time(e1) for e0, e1 in enc_events]
-    if sharded:
-        tt = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
+    all_steps = R.gather(step_ms)                       # [world][steps]
+    per_step_max = [max(r[k] for r in all_steps) for k in range(a.steps)]
+    per_rank_ms = [sum(r) / a.steps for r in all_steps]
+    ms = R.reduce(ms_rank, "max")
     ms_step = ms / a.steps
     value = n_glob / (ms_step / 1e3) / 1e9
 
-    # ---- results of the last step (for CR, roofline bytes and the parity sample)
+    # ---- results of the last step (for CR, roofline bytes and the parity check)
     sizes = ws.sizes[: ws.N].cpu().numpy().view(np.uint32)
     total = int(ws.total.item())
     raw = sizes == C
@@ -577,8 +685,10 @@ def main():
                     f"C=W={C}, m=4, M=259")
         if a.parse != "greedy" or (a.window and a.window != C):
             workload += f", W={a.window or C}, {a.parse} parse"
-    traffic = traffic_from_profiles(workload)
-
+    ent = _profile_entry(workload)
+    par = (f"dp{world} (contiguous chunk shards, {R.backend} all-gather of sizes"
+           + (", ranks share a GPU: functional run, not a scaling number" if R.share_gpu else "") + ")"
+           if sharded else "1 GPU")
     line = {
         "metric": METRIC, "value": round(value, 4), "unit": UNIT, "n_gpus": world,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_step, 4),
@@ -586,35 +696,45 @@ def main():
         "data": "synthetic",
         "config": {"workload": workload, "global_bytes": n_glob, "chunk_size": C, "window": a.window or C,
                    "min_match": 4, "max_match": 259, "parse": a.parse, "chunks_per_gpu": ws.N,
-                   "parallelism": f"dp{world} (contiguous chunk shards, NCCL all-gather of sizes)"
-                   if sharded else "1 GPU",
+                   "parallelism": par,
                    "l2": (f"input ({n_rank >> 20} MiB/GPU) larger than L2 (126 MB); no flush"
                           if n_rank > (126 << 20) else
                           f"input ({n_rank >> 20} MiB/GPU) fits L2; no flush (small config)"),
                    "compression_ratio": round(cr, 4), "raw_chunk_fraction": round(float(raw.mean()), 4)},
+        "step_ms": {"median": round(statistics.median(per_step_max), 4), "min": round(min(per_step_max), 4),
+                    "max": round(max(per_step_max), 4), "mean": round(ms_step, 4),
+                    "what": "per-step device time, max over ranks"},
+        "per_rank_ms": [round(v, 4) for v in per_rank_ms],
+        "rank_spread": round((max(per_rank_ms) - min(per_rank_ms)) / max(per_rank_ms), 4),
         "roofline": {"bound": "hbm", "kernel": "lzr_encode_kernel",
                      "achieved": round(achieved, 3), "peak": hbm_peak, "unit": "GB/s",
                      "frac": round(achieved / hbm_peak, 6),
-                     "traffic": traffic, "peak_source": peak_src,
+                     "traffic": float(ent["dram_bytes_per_launch"]) if ent else None,
+                     "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": enc_algo_bytes,
                      "avg_launch_ms": round(enc_avg_s * 1e3, 4),
-                     "share_of_step": round(statistics.mean(enc_ms) / ms_step, 4),
+                     "share_of_step": round(statistics.mean(enc_ms) / (ms_rank / a.steps), 4),
                      "note": "HBM is the formal roofline of a codec; the encode kernel is "
                              "issue/shared-memory-latency bound (see DESIGN.md and profiles/)"},
         "clocks": clk.summary(),
         "gpu_launches": launches[0],
     }
+    if ent is None:
+        line["roofline"]["profile"] = ("no ncu capture of this workload on this build (kernel-source "
+                                       "hash); limiter / smem pipe / stalls / traffic omitted")
+    else:
+        line["roofline"]["profile"] = {"build": ent.get("build"), "source": ent.get("source")}
     lim = issue_limiter(workload, enc_avg_s, line["clocks"].get("sm_mhz"),
                         torch.cuda.get_device_properties(dev).multi_processor_count)
     if lim:
         line["roofline"]["limiter"] = lim
     # the shared-memory side of the roofline.  (1) the encode
     # kernel's measured shared-memory pipe utilisation (ncu capture of the same
-    # workload); (2) the exhaustive byte-compare ceiling -- one shared-memory
-    # byte per (p, d) cell, (C-1)/2 cells per input byte, 148 SMs x 128 B/clk at
-    # the sampled clock -- which the token-start-only, candidate-exact search is
-    # not bound by (ratio > 1 = faster than any cell-by-cell search could be).
-    ent = _profile_entry(workload)
+    # workload and build); (2) the exhaustive byte-compare ceiling -- one
+    # shared-memory byte per (p, d) cell, (C-1)/2 cells per input byte, 148 SMs x
+    # 128 B/clk at the sampled clock -- which the token-start-only,
+    # candidate-exact search is not bound by (ratio > 1 = faster than any
+    # cell-by-cell search could be).
     sm_mhz = line["clocks"].get("sm_mhz")
     n_sms = torch.cuda.get_device_properties(dev).multi_processor_count
     if sm_mhz:
@@ -622,83 +742,94 @@ def main():
         ceil_gbs = smem_peak / ((C - 1) / 2) / 1e9 * world
         line["roofline"]["smem"] = {
             "pipe_frac": round(ent["smem_pipe_pct"] / 100, 4) if ent and ent.get("smem_pipe_pct") else None,
-            "pipe_source": ent.get("source") if ent else None,
             "peak_TBps": round(smem_peak / 1e12, 2),
             "exhaustive_ceiling_gbs": round(ceil_gbs, 3),
             "value_over_exhaustive_ceiling": round(value / ceil_gbs, 3)}
         if ent and ent.get("stall_share"):
             line["roofline"]["stalls"] = ent["stall_share"]
 
-    # ---- decompression of the same batch, output GB/s
+    # ---- decompression of the same batch, output GB/s of
+    #      the whole job (max over ranks), with a full round-trip compare
     if not a.no_decode:
         dout = torch.empty(n_rank, dtype=torch.uint8, device=dev)
         derr = torch.zeros(1, dtype=torch.int32, device=dev)
         for _ in range(a.warmup):
             lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
-        d0, d1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        d0, d1e = mk(), mk()
         torch.cuda.synchronize()
+        R.barrier()
         d0.record(stream)
         for _ in range(a.steps):
             lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
         d1e.record(stream)
         torch.cuda.synchronize()
-        dms = d0.elapsed_time(d1e) / a.steps
+        dms = R.reduce(d0.elapsed_time(d1e) / a.steps, "max")
         ok = int(derr.item()) == 0 and bool(torch.equal(dout, x))
-        line["decode"] = {"value": round(n_rank / (dms / 1e3) / 1e9, 3), "unit": "GB/s (output)",
-                          "ms_per_step": round(dms, 4), "round_trip": "ok" if ok else "MISMATCH"}
+        ok = R.reduce(0.0 if ok else 1.0, "sum") == 0
+        line["decode"] = {"value": round(n_glob / (dms / 1e3) / 1e9, 3), "unit": "GB/s (output)",
+                          "ms_per_step": round(dms, 4), "round_trip": "ok" if ok else "MISMATCH",
+                          "n_gpus": world}
         del dout
 
-    # ---- end to end through the C ABI with host buffers (pinned), rank 0 view
+    # ---- end to end through the C ABI with host buffers (pinned), every rank
     if not a.no_e2e:
+        import ctypes
+
         n_e2e = min(n_rank, 1 << 30)  # bounded host buffers for the big configs
         hx = x[:n_e2e].cpu().pin_memory()
         scratch = torch.empty(max(256, lzr.lib().lzr_compress_host_scratch_bytes(
-            16 << 20, __import__("ctypes").byref(p.c()))), dtype=torch.uint8, device=dev)
+            16 << 20, ctypes.byref(p.c()))), dtype=torch.uint8, device=dev)
         n_e2e_chunks = -(-n_e2e // C)
         h_out = torch.empty(n_e2e, dtype=torch.uint8, pin_memory=True)
         h_sizes = torch.empty(n_e2e_chunks, dtype=torch.int32, pin_memory=True)
         h_offs = torch.empty(n_e2e_chunks, dtype=torch.int64, pin_memory=True)
         lzr.compress_host(hx, p, 16 << 20, scratch, h_out, h_sizes, h_offs)  # warm-up
         e2e_t = []
+        R.barrier()
         for _ in range(max(1, min(a.steps, 5))):
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             _, _, _, tot = lzr.compress_host(hx, p, 16 << 20, scratch, h_out, h_sizes, h_offs)
             e2e_t.append(time.perf_counter() - t0)
-        e2e_s = statistics.median(e2e_t)
-        e2e_v = n_e2e / e2e_s / 1e9
-        if sharded:
-            tt = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            e2e_v = n_e2e * world / float(tt.item()) / 1e9
+        e2e_s = R.reduce(statistics.median(e2e_t), "max")
+        e2e_v = n_e2e * world / e2e_s / 1e9
         line["e2e"] = {"value": round(e2e_v, 4), "unit": UNIT, "h2d_bytes_per_step": n_e2e,
                        "d2h_bytes_per_step": int(tot) + 12 * n_e2e_chunks,
                        "api": "lzr_compress_host (pinned host in/out, 16 MiB batches, 3 buffer sets, shared H2D / D2H copy streams)"
-                              + ("" if n_e2e == n_rank else f", first {n_e2e >> 20} MiB per GPU")}
+                              + ("" if n_e2e == n_rank else f", first {n_e2e >> 20} MiB per GPU")
+                              + (", per rank; value = all ranks' bytes / slowest rank" if world > 1 else "")}
         del scratch
 
-    if rank == 0 and not a.no_cpu:
-        smp = min(n_rank, (a.cpu_sample_bytes // C) * C) if a.config != 1 else n_rank
-        ns = -(-smp // C)
-        g_offs = ws.offsets[:ns].cpu().numpy().view(np.uint64)
-        end = int(g_offs[-1]) + int(sizes[ns - 1])
-        g_out = ws.out[:end].cpu().numpy()
-        line["cpu_baseline"] = cpu_baseline(x[:smp].cpu().numpy(), p, sizes[:ns], g_offs, g_out,
-                                            smp)
-    if rank == 0 and not a.no_cpu and not a.bytes_per_rank and a.config in (1, 2, 3):
+    # ---- the CPU oracle beside it (rank 0 at N = 1 only): configs 1 and 2 over
+    #      the whole timed stream, bit-exact verdict against the GPU output
+    if world == 1 and not a.no_cpu:
         g_all = ws.out[:total].cpu().numpy()
-        line["cpu_fast"] = cpu_fast(x.cpu().numpy(), p, sizes, g_all)
-        # the paper's GPU-usage decision (§3.2(3) "we compare the compression
-        # performance of the CPU and the GPU to determine when to use the GPU"),
-        # from this run's measured numbers
-        gpu_v = line["value"]
-        e2e_v = line.get("e2e", {}).get("value")
-        cpu_v = line["cpu_fast"]["value"]
-        line["integration"] = {
-            "gpu_device_gbs": gpu_v, "gpu_e2e_gbs": e2e_v, "cpu_fast_gbs": cpu_v,
-            "gpu_over_cpu_e2e": round(e2e_v / cpu_v, 2) if e2e_v else None,
-            "use_gpu_for_compression": bool((e2e_v or gpu_v) > cpu_v),
-            "paper": "GPU 88.3% better than CPU (P:16 §3.2(3), other hardware; context)"}
+        g_offs = ws.offsets[: ws.N].cpu().numpy().view(np.uint64)
+        x_host = x.cpu().numpy()
+        lim_chunks = None if a.config in (1, 2) else max(1, (a.cpu_sample_bytes // C))
+        line["cpu_baseline"] = cpu_baseline(x_host, p, sizes, g_offs, g_all, a.cpu_max_seconds,
+                                            limit_chunks=lim_chunks)
+        if not a.bytes_per_rank and a.config in (1, 2, 3):
+            line["cpu_fast"] = cpu_fast(x_host, p, sizes, g_all)
+            # the paper's GPU-usage decision (§3.2(3) "we compare the compression
+            # performance of the CPU and the GPU to determine when to use the GPU"),
+            # from this run's measured numbers
+            gpu_v = line["value"]
+            e2e_v = line.get("e2e", {}).get("value")
+            cpu_v = line["cpu_fast"]["value"]
+            line["integration"] = {
+                "gpu_device_gbs": gpu_v, "gpu_e2e_gbs": e2e_v, "cpu_fast_gbs": cpu_v,
+                "gpu_over_cpu_e2e": round(e2e_v / cpu_v, 2) if e2e_v else None,
+                "use_gpu_for_compression": bool((e2e_v or gpu_v) > cpu_v),
+                "paper": "GPU 88.3% better than CPU (P:16 §3.2(3), other hardware; context)"}
+    # ---- per class (config 2's "GPU GB/s per class and mix"), this rank's GPU
+    if a.config == 2 and a.cls == "mix" and not a.no_per_class:
+        pc = per_class(lzr, synth, p, n_rank, dev, stream)
+        pc["mix"] = {"compress_gbs": round(n_rank / (ms_rank / a.steps / 1e3) / 1e9, 3),
+                     "compression_ratio": round(cr, 4),
+                     "decompress_gbs": (round(n_rank / (line["decode"]["ms_per_step"] / 1e3) / 1e9, 3)
+                                        if "decode" in line else None)}
+        line["per_class"] = pc
     # the paper's own CPU-vs-GPU compression figures with their hardware (context
     # only: other hardware, no absolute B/s printed)
     line["paper_context"] = {
@@ -708,8 +839,7 @@ def main():
         "gpu_over_cpu": "1.883x (P:16 §3.2(3) '88.3% better')"}
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if sharded:
-        dist.destroy_process_group()
+    R.close()
 
 
 if __name__ == "__main__":

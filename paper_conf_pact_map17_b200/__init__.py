@@ -10,6 +10,7 @@ library has not been built, and the compute calls need a CUDA device.
 """
 from __future__ import annotations
 
+import contextlib
 import ctypes
 import os
 from dataclasses import dataclass
@@ -157,6 +158,29 @@ def _stream(stream, device):
     return ctypes.c_void_p(s.cuda_stream)
 
 
+@contextlib.contextmanager
+def _on(device, stream=None):
+    """Run liblzr calls with `device` current (the C ABI launches on the
+    current device, include/lzr.h) and, when a stream is given, with it as
+    torch's current stream, so that buffers allocated here belong to it and
+    host reads (.item()) synchronise with the work launched on it."""
+    import torch
+
+    with contextlib.ExitStack() as es:
+        dev = torch.device(device) if device is not None else None
+        if dev is not None and dev.type == "cuda":
+            es.enter_context(torch.cuda.device(dev))
+        if stream is not None:
+            es.enter_context(torch.cuda.stream(stream))
+        yield
+
+
+def _same_device(*ts):
+    devs = {t.device for t in ts if t is not None}
+    if len(devs) > 1:
+        raise ValueError(f"tensors on different devices: {sorted(map(str, devs))}")
+
+
 def _require_cuda_u8(t, name):
     import torch
 
@@ -171,13 +195,16 @@ class Workspace:
         import torch
 
         self.n, self.p = n, p
-        dev = torch.device(device) if device is not None else torch.device("cuda")
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
         N = num_chunks(n, p)
-        self.out = torch.empty(max(1, compress_bound(n, p)), dtype=torch.uint8, device=dev)
-        self.sizes = torch.empty(max(1, N), dtype=torch.int32, device=dev)
-        self.offsets = torch.empty(max(1, N), dtype=torch.int64, device=dev)
-        self.total = torch.zeros(1, dtype=torch.int64, device=dev)
-        self.ws = torch.empty(max(256, compress_workspace_bytes(n, p)), dtype=torch.uint8, device=dev)
+        with _on(dev):  # the workspace size depends on the device's SM count
+            self.out = torch.empty(max(1, compress_bound(n, p)), dtype=torch.uint8, device=dev)
+            self.sizes = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+            self.offsets = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+            self.total = torch.zeros(1, dtype=torch.int64, device=dev)
+            self.ws = torch.empty(max(256, compress_workspace_bytes(n, p)), dtype=torch.uint8,
+                                  device=dev)
+        self.device = dev
         self.N = N
 
 
@@ -191,11 +218,13 @@ def compress(t, p: Params = Params(), ws: Workspace | None = None, stream=None):
     """
     _require_cuda_u8(t, "input")
     n = t.numel()
-    if ws is None or ws.n != n or ws.p != p:
-        ws = Workspace(n, p, t.device)
-    st = lib().lzr_compress_chunks(
-        _ptr(t), n, ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
-        _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    with _on(t.device, stream):
+        if ws is None or ws.n != n or ws.p != p:
+            ws = Workspace(n, p, t.device)
+        _same_device(t, ws.ws)
+        st = lib().lzr_compress_chunks(
+            _ptr(t), n, ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
+            _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
     _check(st, "lzr_compress_chunks")
     N = ws.N
     return ws.out, ws.sizes[:N], ws.offsets[:N], ws.total
@@ -203,16 +232,20 @@ def compress(t, p: Params = Params(), ws: Workspace | None = None, stream=None):
 
 def compress_encode(t, p: Params, ws: Workspace, stream=None):
     """Launch only the encode stage (bench timing): sizes in ws.sizes."""
-    st = lib().lzr_compress_encode(_ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.sizes),
-                                   _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    _same_device(t, ws.ws)
+    with _on(t.device, stream):
+        st = lib().lzr_compress_encode(_ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.sizes),
+                                       _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
     _check(st, "lzr_compress_encode")
 
 
 def compress_compact(t, p: Params, ws: Workspace, stream=None):
     """Launch only the scan + compaction stage (after compress_encode)."""
-    st = lib().lzr_compress_compact(
-        _ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
-        _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
+    _same_device(t, ws.ws)
+    with _on(t.device, stream):
+        st = lib().lzr_compress_compact(
+            _ptr(t), t.numel(), ctypes.byref(p.c()), _ptr(ws.out), ws.out.numel(), _ptr(ws.sizes),
+            _ptr(ws.offsets), _ptr(ws.total), _ptr(ws.ws), ws.ws.numel(), _stream(stream, t.device))
     _check(st, "lzr_compress_compact")
 
 
@@ -221,15 +254,17 @@ def scan_sizes(sizes, base: int = 0, offsets=None, total=None, ws=None, stream=N
     import torch
 
     n = sizes.numel()
-    if offsets is None:
-        offsets = torch.empty(max(1, n), dtype=torch.int64, device=sizes.device)
-    if total is None:
-        total = torch.zeros(1, dtype=torch.int64, device=sizes.device)
-    wsb = lib().lzr_scan_workspace_bytes(n)
-    if ws is None or ws.numel() < wsb:
-        ws = torch.empty(max(256, wsb), dtype=torch.uint8, device=sizes.device)
-    st = lib().lzr_scan_sizes(_ptr(sizes), n, base, _ptr(offsets), _ptr(total), _ptr(ws),
-                              ws.numel(), _stream(stream, sizes.device))
+    with _on(sizes.device, stream):
+        if offsets is None:
+            offsets = torch.empty(max(1, n), dtype=torch.int64, device=sizes.device)
+        if total is None:
+            total = torch.zeros(1, dtype=torch.int64, device=sizes.device)
+        wsb = lib().lzr_scan_workspace_bytes(n)
+        if ws is None or ws.numel() < wsb:
+            ws = torch.empty(max(256, wsb), dtype=torch.uint8, device=sizes.device)
+        _same_device(sizes, offsets, total, ws)
+        st = lib().lzr_scan_sizes(_ptr(sizes), n, base, _ptr(offsets), _ptr(total), _ptr(ws),
+                                  ws.numel(), _stream(stream, sizes.device))
     _check(st, "lzr_scan_sizes")
     return offsets[:n], total
 
@@ -241,13 +276,15 @@ def decompress(comp, sizes, offsets, n: int, p: Params = Params(), out=None, err
     import torch
 
     dev = comp.device
-    if out is None:
-        out = torch.empty(max(1, n), dtype=torch.uint8, device=dev)
-    if error is None:
-        error = torch.zeros(1, dtype=torch.int32, device=dev)
-    st = lib().lzr_decompress_chunks(_ptr(comp), _ptr(sizes), _ptr(offsets), n,
-                                     ctypes.byref(p.c()), _ptr(out), _ptr(error),
-                                     _stream(stream, dev))
+    with _on(dev, stream):
+        if out is None:
+            out = torch.empty(max(1, n), dtype=torch.uint8, device=dev)
+        if error is None:
+            error = torch.zeros(1, dtype=torch.int32, device=dev)
+        _same_device(comp, sizes, offsets, out, error)
+        st = lib().lzr_decompress_chunks(_ptr(comp), _ptr(sizes), _ptr(offsets), n,
+                                         ctypes.byref(p.c()), _ptr(out), _ptr(error),
+                                         _stream(stream, dev))
     _check(st, "lzr_decompress_chunks")
     return out[:n], error
 
@@ -291,9 +328,11 @@ def fingerprint(t, chunk_size: int = 4096, out=None, stream=None):
     _require_cuda_u8(t, "input")
     n = t.numel()
     N = -(-n // chunk_size)
-    if out is None:
-        out = torch.empty((max(1, N), 20), dtype=torch.uint8, device=t.device)
-    st = lib().lzr_fingerprint_chunks(_ptr(t), n, chunk_size, _ptr(out), _stream(stream, t.device))
+    with _on(t.device, stream):
+        if out is None:
+            out = torch.empty((max(1, N), 20), dtype=torch.uint8, device=t.device)
+        _same_device(t, out)
+        st = lib().lzr_fingerprint_chunks(_ptr(t), n, chunk_size, _ptr(out), _stream(stream, t.device))
     _check(st, "lzr_fingerprint_chunks")
     return out[:N]
 
@@ -306,10 +345,11 @@ class DedupIndex:
         import torch
 
         self.n_bins, self.bin_slots = n_bins, bin_slots
-        dev = torch.device(device) if device is not None else torch.device("cuda")
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
         nb = lib().lzr_dedup_table_bytes(n_bins, bin_slots)
-        self.table = torch.zeros(max(256, nb), dtype=torch.uint8, device=dev)
-        self.overflow = torch.zeros(1, dtype=torch.int32, device=dev)
+        with _on(dev):
+            self.table = torch.zeros(max(256, nb), dtype=torch.uint8, device=dev)
+            self.overflow = torch.zeros(1, dtype=torch.int32, device=dev)
 
     @classmethod
     def for_chunks(cls, n_chunks: int, device=None, bin_slots: int = 64):
@@ -328,13 +368,15 @@ class DedupIndex:
 
         N = fp.shape[0]
         dev = fp.device
-        if index is None:
-            index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
-        if unique is None:
-            unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
-        st = lib().lzr_dedup_index(_ptr(fp), N, first_chunk, _ptr(self.table), self.n_bins,
-                                   self.bin_slots, _ptr(index), _ptr(unique), _ptr(self.overflow),
-                                   _stream(stream, dev))
+        with _on(dev, stream):
+            if index is None:
+                index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+            if unique is None:
+                unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+            _same_device(fp, self.table, index, unique)
+            st = lib().lzr_dedup_index(_ptr(fp), N, first_chunk, _ptr(self.table), self.n_bins,
+                                       self.bin_slots, _ptr(index), _ptr(unique), _ptr(self.overflow),
+                                       _stream(stream, dev))
         _check(st, "lzr_dedup_index")
         return index[:N], unique[:N]
 
@@ -344,11 +386,13 @@ class DedupIndex:
 
         N = fp.shape[0]
         dev = fp.device
-        index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
-        unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
-        st = lib().lzr_dedup_index_gidx(_ptr(fp), N, _ptr(gidx), _ptr(self.table), self.n_bins,
-                                        self.bin_slots, _ptr(index), _ptr(unique),
-                                        _ptr(self.overflow), _stream(stream, dev))
+        with _on(dev, stream):
+            index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+            unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+            _same_device(fp, gidx, self.table)
+            st = lib().lzr_dedup_index_gidx(_ptr(fp), N, _ptr(gidx), _ptr(self.table), self.n_bins,
+                                            self.bin_slots, _ptr(index), _ptr(unique),
+                                            _ptr(self.overflow), _stream(stream, dev))
         _check(st, "lzr_dedup_index_gidx")
         return index[:N], unique[:N]
 
@@ -358,12 +402,14 @@ def owner_counts(fp, n_owners: int, counts=None, stream=None):
     multi-GPU index (include/lzr.h lzr_dedup_owner_counts)."""
     import torch
 
-    if counts is None:
-        counts = torch.zeros(n_owners, dtype=torch.int32, device=fp.device)
-    else:
-        counts.zero_()
-    st = lib().lzr_dedup_owner_counts(_ptr(fp), fp.shape[0], n_owners, _ptr(counts),
-                                      _stream(stream, fp.device))
+    with _on(fp.device, stream):
+        if counts is None:
+            counts = torch.zeros(n_owners, dtype=torch.int32, device=fp.device)
+        else:
+            counts.zero_()
+        _same_device(fp, counts)
+        st = lib().lzr_dedup_owner_counts(_ptr(fp), fp.shape[0], n_owners, _ptr(counts),
+                                          _stream(stream, fp.device))
     _check(st, "lzr_dedup_owner_counts")
     return counts
 
@@ -375,12 +421,14 @@ def route(fp, first_chunk: int, n_owners: int, base, stream=None):
 
     N = fp.shape[0]
     dev = fp.device
-    cursor = torch.zeros(n_owners, dtype=torch.int32, device=dev)
-    send_fp = torch.empty((max(1, N), 20), dtype=torch.uint8, device=dev)
-    send_gidx = torch.empty(max(1, N), dtype=torch.int64, device=dev)
-    slot = torch.empty(max(1, N), dtype=torch.int32, device=dev)
-    st = lib().lzr_dedup_route(_ptr(fp), N, first_chunk, n_owners, _ptr(base), _ptr(cursor),
-                               _ptr(send_fp), _ptr(send_gidx), _ptr(slot), _stream(stream, dev))
+    with _on(dev, stream):
+        cursor = torch.zeros(n_owners, dtype=torch.int32, device=dev)
+        send_fp = torch.empty((max(1, N), 20), dtype=torch.uint8, device=dev)
+        send_gidx = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+        slot = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+        _same_device(fp, base)
+        st = lib().lzr_dedup_route(_ptr(fp), N, first_chunk, n_owners, _ptr(base), _ptr(cursor),
+                                   _ptr(send_fp), _ptr(send_gidx), _ptr(slot), _stream(stream, dev))
     _check(st, "lzr_dedup_route")
     return send_fp[:N], send_gidx[:N], slot[:N]
 
@@ -391,18 +439,22 @@ def unroute(back, slot, first_chunk: int, stream=None):
 
     N = slot.shape[0]
     dev = slot.device
-    index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
-    unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
-    st = lib().lzr_dedup_unroute(_ptr(back), _ptr(slot), N, first_chunk, _ptr(index), _ptr(unique),
-                                 _stream(stream, dev))
+    with _on(dev, stream):
+        index = torch.empty(max(1, N), dtype=torch.int64, device=dev)
+        unique = torch.empty(max(1, N), dtype=torch.int32, device=dev)
+        _same_device(back, slot)
+        st = lib().lzr_dedup_unroute(_ptr(back), _ptr(slot), N, first_chunk, _ptr(index), _ptr(unique),
+                                     _stream(stream, dev))
     _check(st, "lzr_dedup_unroute")
     return index[:N], unique[:N]
 
 
 def gather_chunks(t, chunk_size: int, unique, rank, out, stream=None):
     """Copy the unique chunks of t to out in stream order (out + rank[i] * C)."""
-    st = lib().lzr_gather_chunks(_ptr(t), t.numel(), chunk_size, _ptr(unique), _ptr(rank), _ptr(out),
-                                 _stream(stream, t.device))
+    _same_device(t, unique, rank, out)
+    with _on(t.device, stream):
+        st = lib().lzr_gather_chunks(_ptr(t), t.numel(), chunk_size, _ptr(unique), _ptr(rank),
+                                     _ptr(out), _stream(stream, t.device))
     _check(st, "lzr_gather_chunks")
     return out
 
@@ -413,25 +465,33 @@ def dedup_compress(t, p: Params = Params(), index: DedupIndex | None = None, fir
     fingerprints, gather the unique chunks, compress them.  Synchronises once to
     size the unique buffer.  Returns a dict with fp, index, unique, rank,
     n_unique, the gathered unique bytes and compress()'s (out, sizes, offsets,
-    total) over them."""
+    total) over them.
+
+    Trust assumption (§3.1(1): the index keys are SHA-1 fingerprints): two
+    chunks with equal SHA-1 are treated as duplicates without a byte compare,
+    as in the paper; a deliberately constructed SHA-1 collision would drop the
+    second chunk's content (R17)."""
     import torch
 
     C = p.chunk_size
-    if index is None:
-        index = DedupIndex.for_chunks(-(-t.numel() // C), t.device)
-    fp = fingerprint(t, C, stream=stream)
-    idx, uniq = index.index(fp, first_chunk, stream=stream)
-    rank, n_uniq_t = scan_sizes(uniq, stream=stream)
-    n = t.numel()
-    N = fp.shape[0]
-    nu = int(n_uniq_t.item())
-    last_unique = N > 0 and bool(uniq[N - 1].item())
-    ubytes = nu * C
-    if last_unique and n % C:
-        ubytes -= C - n % C  # the short tail chunk is the last unique one
-    ubuf = torch.empty(max(1, ubytes), dtype=torch.uint8, device=t.device)
-    gather_chunks(t, C, uniq, rank, ubuf, stream=stream)
-    u = ubuf[:ubytes]
-    out, sizes, offs, total = compress(u, p, ws=ws, stream=stream)
+    # everything below runs on `stream` (and t's device), so the host reads of
+    # the unique count wait for the kernels that produce it
+    with _on(t.device, stream):
+        if index is None:
+            index = DedupIndex.for_chunks(-(-t.numel() // C), t.device)
+        fp = fingerprint(t, C, stream=stream)
+        idx, uniq = index.index(fp, first_chunk, stream=stream)
+        rank, n_uniq_t = scan_sizes(uniq, stream=stream)
+        n = t.numel()
+        N = fp.shape[0]
+        nu = int(n_uniq_t.item())
+        last_unique = N > 0 and bool(uniq[N - 1].item())
+        ubytes = nu * C
+        if last_unique and n % C:
+            ubytes -= C - n % C  # the short tail chunk is the last unique one
+        ubuf = torch.empty(max(1, ubytes), dtype=torch.uint8, device=t.device)
+        gather_chunks(t, C, uniq, rank, ubuf, stream=stream)
+        u = ubuf[:ubytes]
+        out, sizes, offs, total = compress(u, p, ws=ws, stream=stream)
     return {"fp": fp, "index": idx, "unique": uniq, "rank": rank, "n_unique": nu, "unique_bytes": u,
             "out": out, "sizes": sizes, "offsets": offs, "total": total}

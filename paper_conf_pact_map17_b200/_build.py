@@ -28,6 +28,20 @@ def deps():
         os.path.join(ROOT, "include", "lzr.h")]
 
 
+def source_hash() -> str:
+    """Hash of the kernel sources (csrc + include/lzr.h) that liblzr.so is built
+    from: stamps ncu captures so that the bench drops profile-derived keys
+    taken on a different build (no toolchain needed to compute it)."""
+    import hashlib
+
+    h = hashlib.sha256()
+    for d in deps():
+        h.update(os.path.basename(d).encode())
+        with open(d, "rb") as f:
+            h.update(f.read())
+    return h.hexdigest()[:16]
+
+
 def stale() -> bool:
     if not os.path.exists(LIB):
         return True

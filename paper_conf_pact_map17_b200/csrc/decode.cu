@@ -15,7 +15,13 @@
 // only reads bytes before o).  The chunk is written out with 16-byte stores;
 // raw chunks are copied with 16-byte stores from funnel-shifted 4-byte loads.
 // Malformed streams set *err = min(1 + chunk index) (err pre-set to 0x7F7F7F7F,
-// fixed up to 0 afterwards when no chunk was corrupt).
+// fixed up to 0 afterwards when no chunk was corrupt); with err == NULL nothing
+// is reported (include/lzr.h) and the library keeps no global error word.
+// (An output-parallel variant -- each step's output rebuilt in 32-byte windows,
+// lane = byte, token found by a REDUX.OR of the window's token starts, sources
+// by (o - ob) mod d and in-window pointer jumping, stream staged in shared
+// memory -- measured no faster: text 230-248 vs 243 GB/s, zero-runs 318-395 vs
+// 677.)
 #include <mutex>
 
 #include "lzr_internal.cuh"
@@ -27,8 +33,6 @@ namespace {
 constexpr int kDecWarpsMax = 16;
 constexpr int32_t kNoError = 0x7F7F7F7F;
 constexpr uint32_t kLaneCopyMax = 16;  // matches up to this length: one lane, byte-serial
-
-__device__ int32_t g_scratch_err;
 
 // Word i of the aligned view of src - mis, reading only bytes in [mis, mis + len)
 // (edge words byte by byte, so no access leaves the caller's buffer).
@@ -171,7 +175,7 @@ __global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
     }
     if (!bad && ip != S) bad = true;
     if (bad) {
-      if (lane == 0) atomicMin(err, (int32_t)(c + 1));
+      if (lane == 0 && err) atomicMin(err, (int32_t)(c + 1));
       __syncwarp();
       continue;
     }
@@ -215,39 +219,41 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   if (warps > LZR_DEC_WARPS) warps = LZR_DEC_WARPS;
   if (warps < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)warps * stride;
-  // smem attribute + occupancy at this size, cached per device (host calls
-  // kept off the per-launch path)
-  static size_t c_smem[64] = {};
-  static int c_per_sm[64] = {};
+  // The dynamic shared-memory limit is raised once per device to the opt-in
+  // maximum (never lowered, so concurrent callers with different chunk sizes
+  // cannot undercut each other); the occupancy is cached per smem size.
+  struct Cached {
+    bool attr;
+    size_t smem;
+    int per_sm;
+  };
+  static Cached cache[64] = {};
   static std::mutex mu;
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   int per_sm = 0;
   {
     std::lock_guard<std::mutex> lk(mu);
-    if (dev >= 0 && dev < 64 && c_smem[dev] == smem) per_sm = c_per_sm[dev];
+    if (!cache[dev].attr) {
+      e = cudaFuncSetAttribute(lzr_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
+      if (e != cudaSuccess) return e;
+      cache[dev].attr = true;
+    }
+    if (cache[dev].smem == smem) per_sm = cache[dev].per_sm;
   }
   if (per_sm == 0) {
-    e = cudaFuncSetAttribute(lzr_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     // (LZR_DEC_ONEWAVE: at most one resident wave of CTAs, warps loop over chunks)
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel, warps * 32, smem);
     if (e != cudaSuccess || per_sm < 1) per_sm = 1;
     std::lock_guard<std::mutex> lk(mu);
-    if (dev >= 0 && dev < 64) {
-      c_smem[dev] = smem;
-      c_per_sm[dev] = per_sm;
-    }
+    cache[dev].smem = smem;
+    cache[dev].per_sm = per_sm;
   }
   int32_t* errp = err;
   if (errp) {
     e = cudaMemsetAsync(errp, 0x7F, sizeof(int32_t), s);
-    if (e != cudaSuccess) return e;
-  }
-  // a private error word is needed when the caller passes none
-  if (!errp) {
-    e = cudaGetSymbolAddress((void**)&errp, g_scratch_err);
     if (e != cudaSuccess) return e;
   }
   size_t blocks = (N + warps - 1) / warps;

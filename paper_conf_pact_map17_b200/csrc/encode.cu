@@ -1078,10 +1078,13 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   if (groups > 15) groups = 15;  // named barriers 1..15
   if (groups < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)groups * a.L.per_group;
-  // the smem attribute and the occupancy of this instantiation at this smem
-  // size, per device: host calls cached so that batch-by-batch callers (the
-  // host pipeline) do not pay them on every launch
+  // Host calls cached per device so that batch-by-batch callers (the host
+  // pipeline) do not pay them on every launch.  The dynamic shared-memory limit
+  // of this instantiation is raised once to the device's opt-in maximum and
+  // never lowered, so concurrent callers with different chunk sizes cannot
+  // undercut each other's launch; the occupancy is cached per smem size.
   struct Cached {
+    bool attr;
     size_t smem;
     int per_sm;
   };
@@ -1090,15 +1093,19 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   int dev = 0;
   cudaError_t err = cudaGetDevice(&dev);
   if (err != cudaSuccess) return err;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
   int per_sm = 0;
   {
     std::lock_guard<std::mutex> lk(mu);
-    if (dev >= 0 && dev < 64 && cache[dev].smem == smem) per_sm = cache[dev].per_sm;
+    if (!cache[dev].attr) {
+      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
+      if (err != cudaSuccess) return err;
+      cache[dev].attr = true;
+    }
+    if (cache[dev].smem == smem) per_sm = cache[dev].per_sm;
   }
   if (per_sm == 0) {
-    err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
-                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (err != cudaSuccess) return err;
     // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
     if (MinBlocks<K, G1>::value > 1 &&
@@ -1107,7 +1114,8 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
       per_sm = 1;
     if (per_sm < 1) per_sm = 1;
     std::lock_guard<std::mutex> lk(mu);
-    if (dev >= 0 && dev < 64) cache[dev] = {smem, per_sm};
+    cache[dev].smem = smem;
+    cache[dev].per_sm = per_sm;
   }
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);

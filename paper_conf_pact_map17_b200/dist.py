@@ -18,6 +18,7 @@ offset logic over a gloo group; there is no CPU fallback in the product path.
 """
 from __future__ import annotations
 
+from contextlib import nullcontext
 from dataclasses import dataclass
 
 import torch
@@ -38,27 +39,73 @@ def max_shard(n_chunks: int, world: int) -> int:
     return -(-n_chunks // world)
 
 
+def _staged(group) -> bool:
+    """True when the group's backend cannot take CUDA tensors in the exchange
+    collectives (gloo): the tensors are then staged through host memory.  The
+    data-path backend of the product is NCCL; gloo serves several ranks that
+    share one GPU (tests, bench --backend gloo)."""
+    return dist.get_backend(group) != "nccl"
+
+
+def all_gather_into(out: torch.Tensor, inp: torch.Tensor, group=None) -> None:
+    """all_gather_into_tensor on NCCL; host-staged all_gather on gloo."""
+    if not _staged(group) or not out.is_cuda:
+        try:
+            dist.all_gather_into_tensor(out, inp, group=group)
+            return
+        except (RuntimeError, NotImplementedError):
+            if out.is_cuda:
+                raise
+    o = torch.empty(out.shape, dtype=out.dtype)
+    dist.all_gather(list(o.chunk(dist.get_world_size(group))), inp.cpu(), group=group)
+    out.copy_(o)
+
+
+def all_to_all_into(out: torch.Tensor, inp: torch.Tensor, out_splits, in_splits, group=None) -> None:
+    """all_to_all_single on NCCL; host-staged on gloo."""
+    if not _staged(group) or not out.is_cuda:
+        dist.all_to_all_single(out, inp, output_split_sizes=out_splits,
+                               input_split_sizes=in_splits, group=group)
+        return
+    o = torch.empty(out.shape, dtype=out.dtype)
+    dist.all_to_all_single(o, inp.cpu(), output_split_sizes=out_splits,
+                           input_split_sizes=in_splits, group=group)
+    out.copy_(o)
+
+
+def _on(device):
+    """Make `device` current around liblzr calls (the C ABI works on the
+    current device, include/lzr.h)."""
+    dev = torch.device(device) if device is not None else None
+    return torch.cuda.device(dev) if dev is not None and dev.type == "cuda" else nullcontext()
+
+
 class CudaOps:
     """The product path: liblzr kernels + torch.distributed collectives."""
 
     def __init__(self, p: Params, n_local: int, device):
         self.p = p
-        self.ws = Workspace(n_local, p, device)
+        self.device = device
+        with _on(device):
+            self.ws = Workspace(n_local, p, device)
 
     def bind_sizes(self, sizes_pad):
         # the encoder writes the per-chunk sizes straight into the padded
         # all-gather input (no copy on the data path)
+        assert sizes_pad.numel() >= self.ws.N
         self.ws.sizes = sizes_pad
 
     def compress(self, x):
-        out, sizes, offsets, total = compress(x, self.p, ws=self.ws)
+        with _on(x.device):
+            out, sizes, offsets, total = compress(x, self.p, ws=self.ws)
         return out, sizes, total
 
     def scan(self, sizes_all, offsets, total):
-        scan_sizes(sizes_all, 0, offsets=offsets, total=total)
+        with _on(sizes_all.device):
+            scan_sizes(sizes_all, 0, offsets=offsets, total=total)
 
     def all_gather(self, out, inp, group):
-        dist.all_gather_into_tensor(out, inp, group=group)
+        all_gather_into(out, inp, group)
 
 
 @dataclass
@@ -69,13 +116,14 @@ class ShardResult:
     sizes_all: torch.Tensor      # [R * maxN] int32, zero-padded per rank
     offsets_all: torch.Tensor    # [R * maxN] int64 global exclusive offsets
     global_total: torch.Tensor   # [1] int64
-    lo: int
+    lo: int                      # this rank's chunk range [lo, hi) of the global stream
     hi: int
-    max_n: int
+    max_n: int                   # padded shard length (ceil(N / R))
+    rank: int                    # this rank in the group (row of sizes_all / offsets_all)
 
     def global_offsets(self) -> torch.Tensor:
         """Global offsets of this rank's chunks (view)."""
-        r = self.lo_rank
+        r = self.rank
         return self.offsets_all[r * self.max_n: r * self.max_n + (self.hi - self.lo)]
 
 
@@ -118,10 +166,8 @@ class ShardedCompressor:
             total = torch.zeros(1, dtype=torch.int64, device=self.sizes_pad.device)
         self.ops.all_gather(self.sizes_all, self.sizes_pad, self.group)
         self.ops.scan(self.sizes_all, self.offsets_all, self.global_total)
-        res = ShardResult(out, sizes[:nl], total, self.sizes_all, self.offsets_all,
-                          self.global_total, self.lo, self.hi, self.max_n)
-        res.lo_rank = self.rank
-        return res
+        return ShardResult(out, sizes[:nl], total, self.sizes_all, self.offsets_all,
+                           self.global_total, self.lo, self.hi, self.max_n, self.rank)
 
 
 def compress_sharded(x_local, p: Params, n_bytes_global: int, group=None):
@@ -137,23 +183,27 @@ class CudaDedupOps:
         self.index = index
 
     def fingerprint(self, x, C):
-        return fingerprint(x, C)
+        with _on(x.device):
+            return fingerprint(x, C)
 
     def owner_counts(self, fp, R):
-        return owner_counts(fp, R)
+        with _on(fp.device):
+            return owner_counts(fp, R)
 
     def route(self, fp, first, R, base):
-        return route(fp, first, R, base)
+        with _on(fp.device):
+            return route(fp, first, R, base)
 
     def index_gidx(self, fp, gidx):
-        return self.index.index_gidx(fp, gidx)[0]
+        with _on(fp.device):
+            return self.index.index_gidx(fp, gidx)[0]
 
     def unroute(self, back, slot, first):
-        return unroute(back, slot, first)
+        with _on(slot.device):
+            return unroute(back, slot, first)
 
     def all_to_all(self, out, inp, out_splits, in_splits, group):
-        dist.all_to_all_single(out, inp, output_split_sizes=out_splits,
-                               input_split_sizes=in_splits, group=group)
+        all_to_all_into(out, inp, out_splits, in_splits, group)
 
 
 class ShardedDedup:
@@ -179,7 +229,8 @@ class ShardedDedup:
         if ops is None:
             # an owner receives ~n_local chunks on average; skew covers imbalance
             cap = int(skew * max(1, n_local_max)) + 1024
-            ops = CudaDedupOps(DedupIndex.for_chunks(cap, device, bin_slots))
+            with _on(device):
+                ops = CudaDedupOps(DedupIndex.for_chunks(cap, device, bin_slots))
         self.ops = ops
 
     def __call__(self, x_local, chunk_size: int, first_chunk: int):

@@ -129,3 +129,180 @@ def test_dedup_routing_kernels_emulated_ranks(ref):
     r_idx, r_hit, _ = ref.dedup_index(ref.fingerprints(x.cpu().numpy(), C), 0)
     assert np.array_equal(np.concatenate(got_i).view(np.uint64), r_idx)
     assert np.array_equal(np.concatenate(got_u).astype(bool), ~r_hit.astype(bool))
+
+
+# ---- several ranks on the real kernels ---------------------------------------
+# The pool gives one GPU per call, and NCCL refuses two ranks on one device, so
+# these run R processes on cuda:0 over a gloo group: the product ops (CudaOps /
+# CudaDedupOps: liblzr kernels) with the exchange tensors staged through host
+# memory (dist.all_gather_into / all_to_all_into).  Uneven shards exercise the
+# zero padding of the size all-gather and the global scan over R * ceil(N/R).
+def _mp_compress_worker(rank, world, port, n_global, C, parse, q):
+    import torch.distributed as dist
+
+    import synth
+    import paper_conf_pact_map17_b200 as lzr
+    from paper_conf_pact_map17_b200.dist import ShardedCompressor
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        p = lzr.Params(chunk_size=C, parse=parse)
+        sc = ShardedCompressor(n_global, p, None, dev)
+        x = torch.empty(sc.n_local, dtype=torch.uint8, device=dev)
+        if sc.n_local:
+            synth.fill_device(x, C, "mix", first_chunk=sc.lo)
+        res = sc(x)
+        torch.cuda.synchronize()
+        lt = int(res.local_total.item())
+        q.put((rank, sc.lo, sc.hi, sc.max_n, res.rank, res.global_offsets().cpu().numpy().copy(),
+               int(res.global_total.item()), res.out[:lt].cpu().numpy().copy(),
+               res.local_sizes.cpu().numpy().copy(), res.sizes_all.cpu().numpy().copy()))
+    except Exception as e:  # surface the failure to the parent
+        q.put((rank, repr(e)))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def _spawn(target, world, args, timeout=300):
+    import torch.multiprocessing as mp
+
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=target, args=(r, world, port, *args, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = [q.get(timeout=timeout) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=60)
+    for r in res:
+        assert len(r) > 2, f"rank {r[0]} failed: {r[1]}"
+    for pr in procs:
+        assert pr.exitcode == 0
+    return sorted(res, key=lambda t: t[0])
+
+
+@pytest.mark.parametrize("world,nchunks,tail,C,parse", [(2, 301, 123, 4096, 0), (3, 100, 0, 4096, 0),
+                                                       (3, 7, 5, 8192, 0), (2, 55, 77, 4096, 1),
+                                                       (4, 3, 0, 4096, 0)])
+def test_sharded_real_kernels_multirank(ref, world, nchunks, tail, C, parse):
+    """ShardedCompressor with the CUDA ops at world 2-4 (uneven shards, a rank
+    with no chunk at world 4 / 3 chunks) == the oracle over the whole stream:
+    global offsets, total, gathered sizes and every rank's compacted bytes."""
+    import __graft_entry__
+    __graft_entry__.build()
+    import synth
+    from paper_conf_pact_map17_b200.dist import max_shard, shard_range
+
+    n_global = nchunks * C + tail
+    res = _spawn(_mp_compress_worker, world, (n_global, C, parse))
+    x = synth.fill_host(n_global, C, "mix")
+    r_out, r_sizes, r_offs, r_tot = ref.compress(x, ref.Params(chunk_size=C, parse=parse))
+    N = r_sizes.size
+    mx = max_shard(N, world)
+    for rank, lo, hi, max_n, rrank, goffs, gtot, out_local, lsizes, sizes_all in res:
+        assert (lo, hi) == shard_range(N, world, rank) and rrank == rank and max_n == mx
+        assert gtot == r_tot
+        assert np.array_equal(goffs.view(np.uint64), r_offs[lo:hi])
+        assert np.array_equal(lsizes.view(np.uint32), r_sizes[lo:hi])
+        if hi > lo:
+            a = int(r_offs[lo])
+            assert out_local.tobytes() == r_out[a: a + out_local.size].tobytes()
+        sa = sizes_all.view(np.uint32)
+        got = np.concatenate([sa[r * mx: r * mx + (shard_range(N, world, r)[1] - shard_range(N, world, r)[0])]
+                              for r in range(world)])
+        assert np.array_equal(got, r_sizes)
+        pads = np.concatenate([sa[r * mx + (shard_range(N, world, r)[1] - shard_range(N, world, r)[0]):(r + 1) * mx]
+                               for r in range(world)])
+        assert not pads.any()
+
+
+def _mp_dedup_worker(rank, world, port, n_chunks, C, rounds, q):
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_pact_map17_b200.dist import ShardedDedup, shard_range
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        xh = synth.fill_host(n_chunks * C, C, "mix_dedup")
+        per = -(-n_chunks // rounds)
+        sd = ShardedDedup(per, device=dev)
+        outs = []
+        for b in range(rounds):
+            g0, g1 = b * per, min(n_chunks, (b + 1) * per)
+            lo, hi = shard_range(g1 - g0, world, rank)
+            lo, hi = g0 + lo, g0 + hi
+            x = torch.from_numpy(np.ascontiguousarray(xh[lo * C:hi * C])).to(dev)
+            _, idx, un = sd(x, C, lo)
+            torch.cuda.synchronize()
+            outs.append((lo, idx.cpu().numpy().copy(), un.cpu().numpy().copy()))
+        assert int(sd.ops.index.overflow.item()) == 0
+        q.put((rank, outs, None))
+    except Exception as e:
+        q.put((rank, repr(e)))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,rounds", [(2, 1), (3, 2)])
+def test_sharded_dedup_real_kernels_multirank(ref, world, rounds):
+    """ShardedDedup with the CUDA ops at world 2-3: fingerprints routed to their
+    owner rank, owner-side insert-or-min, index numbers back; == single-process
+    first-occurrence indexing of the whole stream (R18)."""
+    import __graft_entry__
+    __graft_entry__.build()
+    import synth
+
+    C, n_chunks = 4096, 1500
+    res = _spawn(_mp_dedup_worker, world, (n_chunks, C, rounds))
+    x = synth.fill_host(n_chunks * C, C, "mix_dedup")
+    r_idx, r_hit, _ = ref.dedup_index(ref.fingerprints(x, C), 0)
+    got_idx = np.zeros(n_chunks, np.int64) - 1
+    got_un = np.zeros(n_chunks, np.int32) - 1
+    for rank, outs, _ in res:
+        for b0, idx, un in outs:
+            got_idx[b0:b0 + len(idx)] = idx
+            got_un[b0:b0 + len(un)] = un
+    assert np.array_equal(got_idx.astype(np.uint64), r_idx)
+    assert np.array_equal(got_un.astype(bool), ~r_hit.astype(bool))
+
+
+def _bench_line(args, timeout=900):
+    import json
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), *args], capture_output=True,
+                       text=True, timeout=timeout, cwd=root)
+    assert r.returncode == 0, r.stderr[-3000:]
+    return json.loads(r.stdout.strip().splitlines()[-1])
+
+
+def test_bench_gpus2_self_launch_gloo():
+    """`bench.py --gpus 2` without torchrun starts 2 ranks itself (gloo, both on
+    the one GPU): the line says n_gpus 2, covers both shards, round trip ok."""
+    d = _bench_line(["--gpus", "2", "--backend", "gloo", "--bytes-per-rank", str(16 << 20),
+                     "--steps", "3", "--warmup", "3", "--no-cpu", "--no-e2e", "--no-per-class"])
+    assert d["n_gpus"] == 2 and len(d["per_rank_ms"]) == 2
+    assert d["config"]["global_bytes"] == 2 * (16 << 20)
+    assert d["decode"]["round_trip"] == "ok"
+    assert "dp2" in d["config"]["parallelism"]
+
+
+def test_bench_config5_gpus2_gloo():
+    d = _bench_line(["--config", "5", "--gpus", "2", "--backend", "gloo", "--bytes-per-rank",
+                     str(32 << 20), "--steps", "3", "--warmup", "3", "--no-cpu"])
+    assert d["n_gpus"] == 2 and len(d["per_rank_ms"]) == 2
+    assert 1.8 < d["config"]["dedup_ratio"] < 2.2

@@ -369,3 +369,39 @@ def test_compress_host_concurrent_callers(lzr, ref):
         assert np.array_equal(h_sizes.numpy().view(np.uint32), g_sizes)
         assert np.array_equal(h_offs.numpy().view(np.uint64), g_offs)
         assert np.array_equal(h_out[:tot].numpy(), g_out)
+
+
+def test_decode_without_error_word(lzr):
+    """d_error == NULL through the C ABI: the stream still decodes (nothing is
+    reported; the library keeps no error word of its own, include/lzr.h)."""
+    import ctypes
+
+    x = synth.fill_host(1 << 20, 4096, "mix", seed=3)
+    p = lzr.Params()
+    xd = torch.from_numpy(x).cuda()
+    out, sizes, offs, total = lzr.compress(xd, p)
+    y = torch.empty_like(xd)
+    st = lzr.lib().lzr_decompress_chunks(
+        lzr._ptr(out), lzr._ptr(sizes), lzr._ptr(offs), x.size, ctypes.byref(p.c()), lzr._ptr(y),
+        ctypes.c_void_p(0), ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    assert st == 0
+    torch.cuda.synchronize()
+    assert torch.equal(y, xd)
+
+
+def test_other_stream_dedup_and_compress(lzr, ref):
+    """dedup_compress / compress on a non-default stream size their
+    buffers from values produced on that stream (no stale host reads)."""
+    x = synth.fill_host(4 << 20, 4096, "mix_dedup", seed=5)
+    xd = torch.from_numpy(x).cuda()
+    s = torch.cuda.Stream()
+    p = lzr.Params()
+    for _ in range(3):
+        res = lzr.dedup_compress(xd, p, stream=s)
+        s.synchronize()
+        r_idx, r_hit, _ = ref.dedup_index(ref.fingerprints(x, 4096), 0)
+        assert res["n_unique"] == int((r_hit == 0).sum())
+        ub = np.concatenate([x[i * 4096:(i + 1) * 4096] for i in np.flatnonzero(r_hit == 0)])
+        r_out, _, _, r_tot = ref.compress(ub, ref.Params())
+        assert int(res["total"].item()) == r_tot
+        assert np.array_equal(res["out"][:r_tot].cpu().numpy(), r_out)

@@ -1,5 +1,6 @@
 """Build liblzr variants for A/B timing: python tools/build_variant.py NAME file.cu [-DX ...]
-(the named encode.cu replaces csrc/encode.cu in a temp copy; output paper_conf_pact_map17_b200/liblzr_NAME.so)"""
+(file.cu replaces the csrc file of the same base name -- encode.cu unless the
+name is one of csrc's -- in a temp copy; output paper_conf_pact_map17_b200/liblzr_NAME.so)"""
 import os, shutil, subprocess, sys, tempfile
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_pact_map17_b200 import _build
@@ -8,7 +9,8 @@ extra = sys.argv[3:]
 tmp = tempfile.mkdtemp()
 src = os.path.join(tmp, "csrc")
 shutil.copytree(_build.CSRC, src)
-shutil.copy(enc, os.path.join(src, "encode.cu"))
+base = os.path.basename(enc)
+shutil.copy(enc, os.path.join(src, base if os.path.exists(os.path.join(src, base)) else "encode.cu"))
 inc = os.path.join(os.path.dirname(tmp), "include")
 srcs = sorted(os.path.join(src, f) for f in os.listdir(src) if f.endswith(".cu"))
 out = os.path.join(_build.PKG, f"liblzr_{name}.so")

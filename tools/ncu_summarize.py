@@ -3,6 +3,8 @@ usage: python tools/ncu_summarize.py r01"""
 import csv, io, json, os, subprocess, sys
 R = sys.argv[1] if len(sys.argv) > 1 else "r01"
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+from paper_conf_pact_map17_b200._build import source_hash  # noqa: E402
 out = {}
 # launch list -> per-kernel share
 rows = list(csv.reader(open(os.path.join(ROOT, "gpurun_out", f"launches_{R}.csv"))))
@@ -49,7 +51,9 @@ out["encode_full"] = full
 workload = "cfg2: 256 MiB mix per GPU, C=W=4096, m=4, M=259"
 summ_path = os.path.join(ROOT, "profiles", "encode_ncu_summary.json")
 summ = json.load(open(summ_path)) if os.path.exists(summ_path) else {}
-summ[workload] = {"round": R, "dram_bytes_per_launch": full["dram_bytes_per_launch"],
+bpath = os.path.join(ROOT, "gpurun_out", f"build_{R}.txt")
+build = open(bpath).read().strip() if os.path.exists(bpath) else source_hash()
+summ[workload] = {"round": R, "build": build, "dram_bytes_per_launch": full["dram_bytes_per_launch"],
                   "duration_s": full.get("gpu__time_duration.sum"),
                   "warp_inst_per_launch": full.get("smsp__inst_executed.sum"),
                   "ipc": full.get("sm__inst_executed.avg.per_cycle_active"),
