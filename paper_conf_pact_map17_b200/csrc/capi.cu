@@ -53,6 +53,7 @@ uint32_t enc_warps_per_chunk(uint32_t C) {
     const char* e = getenv("LZR_ENCODE_WARPS");
     env = (e && ((*e >= '1' && *e <= '4') || *e == '8')) ? (*e - '0') : 0;
   }
+  if (C > kBigChunk) return 16u;  // the big-chunk layout (lzr_internal.cuh) is built for 16
   if (env > 0) return (uint32_t)env;
   return C > 4096 ? 8u : (C >= 1024 ? 4u : 1u);
 }
@@ -67,6 +68,7 @@ uint32_t enc_scatter_splits(uint32_t K) {
   }
   // default (config-3 sweep, 1 x B200): 1 split at K = 4 (C = 4 KiB: the full
   // C-bucket table matters more than the serial scatter), 4 at K = 8
+  if (K > 8) return 1u;  // big chunks: one scatter (their B counters fill the slot region)
   const uint32_t ns = env > 0 ? (uint32_t)env : (K >= 8 ? 4u : 1u);
   return K < 4 ? 1u : (ns < K ? ns : K);  // (kernels are instantiated for these)
 }
@@ -79,14 +81,21 @@ WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
   const size_t N = (n_bytes + C - 1) / C;
   DevInfo di;
   const size_t sms = dev_info(&di) == cudaSuccess ? (size_t)di.sm_count : 1024;
-  // resident chunk groups: grid (<= SMs) x groups per CTA (<= 16); the launch
-  // uses at most ceil(N / groups) CTAs, i.e. at most N + 15 groups
-  size_t groups = sms * kMaxGroupsPerSm;
+  // resident chunk groups: grid (<= SMs x CTAs per SM) x groups per CTA; both
+  // bounded by one SM's shared memory (228 KB) over a group's footprint, and
+  // by 16 per SM; the launch uses at most ceil(N / groups) CTAs, i.e. at most
+  // N + 15 groups
+  const uint32_t K = enc_warps_per_chunk((uint32_t)C);
+  const EncLayout L = enc_layout((uint32_t)C, K, enc_scatter_splits(K));
+  size_t per_sm = kSmemPerSm / L.per_group;
+  if (per_sm > kMaxGroupsPerSm) per_sm = kMaxGroupsPerSm;
+  if (per_sm < 1) per_sm = 1;
+  size_t groups = sms * per_sm;
   if (groups > N + kMaxGroupsPerSm) groups = N + kMaxGroupsPerSm;
   w.ctrl_off = 0;
   w.slots_off = 256;
   w.scratch_off = w.slots_off + align_up_z(N * C, 256);
-  w.scan_off = w.scratch_off + align_up_z(groups * 2 * C, 256);
+  w.scan_off = w.scratch_off + align_up_z(groups * enc_scratch_per_group(L, (uint32_t)C), 256);
   w.total = w.scan_off + scan_ws_bytes(N);
   return w;
 }
@@ -167,9 +176,9 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
   const uint32_t K = enc_warps_per_chunk(p->chunk_size);
   a.L = enc_layout(p->chunk_size, K, enc_scatter_splits(K));
-  // positions are 15-bit in the index (bit 15 marks bucket starts) and one
-  // chunk's index must fit one CTA's shared memory
-  if (p->chunk_size > 32768 || (int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;
+  // one chunk's index must fit one CTA's shared memory (C <= 32 KiB: 15-bit
+  // positions + bucket-start marks; above: the big-chunk layout)
+  if ((int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;
   uint8_t* ws = (uint8_t*)d_workspace;
   a.slots = ws + w.slots_off;
   a.scratch = ws + w.scratch_off;

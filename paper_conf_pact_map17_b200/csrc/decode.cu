@@ -217,6 +217,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
 #endif
   int warps = smem_optin / (int)stride;
   if (warps > LZR_DEC_WARPS) warps = LZR_DEC_WARPS;
+  if (C > 16384) warps = 1;  // one chunk per CTA: more CTAs fit an SM
   if (warps < 1) return cudaErrorInvalidConfiguration;
   const size_t smem = (size_t)warps * stride;
   // The dynamic shared-memory limit is raised once per device to the opt-in

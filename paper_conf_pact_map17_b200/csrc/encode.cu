@@ -90,6 +90,16 @@ __device__ __forceinline__ void red_or_if(bool pred, uint32_t* addr, uint32_t v)
       "r"(smem_u32(addr)), "r"(v)
       : "memory");
 }
+// token-start bits of a walk segment: shared memory, or (big chunks) the
+// group's global scratch
+template <bool BIG>
+__device__ __forceinline__ void tb_or_if(bool pred, uint32_t* addr, uint32_t v) {
+  if (BIG) {
+    if (pred) atomicOr(addr, v);
+  } else {
+    red_or_if(pred, addr, v);
+  }
+}
 // predicated 16-bit global store
 __device__ __forceinline__ void st_u16_if(bool pred, uint16_t* addr, uint32_t v) {
   asm volatile(
@@ -185,7 +195,7 @@ struct Smem {
   uint32_t* cb;      // 1: byte differs from the previous one (run boundaries);
                      // after the walk: match bit per token index (flag bytes)
   uint32_t* tb;      // K token-start bitmaps, one per walk segment
-  uint32_t* runs;    // (end << 16) | start of every run of >= k equal bytes
+  uint32_t* runs;    // ((end - 1) << 16) | start of every run of >= k equal bytes
   uint32_t* ctrl;    // chunk, U, nruns, prog[K], sync[K], T[K], M[K]
   uint64_t* bar;
 };
@@ -212,7 +222,7 @@ __device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, u
     uint32_t pk = 0;
     if (j < nruns) {
       const uint32_t rr = S.runs[j];
-      const uint32_t st = rr & 0xFFFFu, e = rr >> 16;
+      const uint32_t st = rr & 0xFFFFu, e = (rr >> 16) + 1u;  // run [st, e)
       if (data[st] == b) {
         const bool reach = e - st >= r;
         const uint32_t q = reach ? e - r : st;
@@ -232,6 +242,7 @@ __device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, u
 // the generic path then evaluates only candidates that also match the byte at
 // offset floor; the result is exact whenever it exceeds floor (every candidate
 // reaching the maximum passes that test), otherwise it is some value <= floor.
+template <bool BIG>
 __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32_t n,
                                                uint32_t nruns, const EncArgs& a, uint32_t lane,
                                                uint32_t floor = 0) {
@@ -259,17 +270,40 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
     pw[2] = __funnelshift_r(a2, a3, sa);
     pw[3] = __funnelshift_r(a3, a4, sa);
   }
-  for (int sb = (int)S.slot[p] - 1;; sb -= 32) {  // the walk only asks at positions with a candidate
+  // p's own index entry (the walk only asks at positions with a candidate, so
+  // p is indexed); the candidates are the entries of its bucket below it
+  int sb0, bstart = 0;
+  if (BIG) {
+    // big chunks: no slot array -- find p inside its bucket [bs, be) (entries
+    // ascending) by a 32-ary search, lane i probing lo + i * step
+    const uint16_t* ends = S.slot;
+    const uint32_t h = khash(kp, a.L.hbits, a.kmask);
+    const uint32_t bs = h ? ends[h - 1] : 0u;
+    uint32_t lo = bs, hi = ends[h];  // p in [lo, hi), sorted[lo] <= p
+    while (hi - lo > 32u) {
+      const uint32_t step = (hi - lo + 31u) >> 5;
+      const uint32_t idx = lo + lane * step;
+      const uint32_t bal = __ballot_sync(kFull, idx < hi && S.sorted[idx] <= p);
+      lo += (31u - __clz(bal)) * step;
+      hi = min(hi, lo + step);
+    }
+    const uint32_t bal = __ballot_sync(kFull, lo + lane < hi && S.sorted[lo + lane] <= p);
+    sb0 = (int)(lo + 31u - __clz(bal));
+    bstart = (int)bs;
+  } else {
+    sb0 = (int)S.slot[p];
+  }
+  for (int sb = sb0 - 1;; sb -= 32) {
     const int s = sb - (int)lane;
     uint32_t e = kFirst, q = 0;
-    bool ok = s >= 0;
+    bool ok = s >= bstart;
     if (ok) {
       e = S.sorted[s];
-      q = e & kPos;
+      q = BIG ? e : e & kPos;
       ok = all_in_window || p - q <= a.W;
     }
     // lanes up to and including the bucket's first entry, and inside the window
-    const uint32_t m_first = __ballot_sync(kFull, ok && (e & kFirst));
+    const uint32_t m_first = BIG ? 0u : __ballot_sync(kFull, ok && (e & kFirst));
     const uint32_t m_stop = __ballot_sync(kFull, !ok);
     uint32_t lim = 32;
     if (m_first) lim = (uint32_t)__ffs(m_first);
@@ -311,7 +345,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 #ifndef LZR_PUB
 #define LZR_PUB 64  // progress published every LZR_PUB bytes of parse
 #endif
-template <int K, bool LZ>
+template <int K, bool LZ, bool BIG>
 __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
                                              uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
                                              const EncArgs& a, uint32_t lane) {
@@ -346,7 +380,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
 #ifdef LZR_PHASE_TIMING
       const long long tb0 = clock64();
 #endif
-      r = (LZ && q == cq) ? cr : best_match(S, q, n, nruns, a, lane);
+      r = (LZ && q == cq) ? cr : best_match<BIG>(S, q, n, nruns, a, lane);
 #ifdef LZR_PHASE_TIMING
       t_bm += clock64() - tb0;
       ++n_bm;
@@ -355,7 +389,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       // LZ: a longer match at q + 1 is possible only if l is below its cap
       // min(M, n - q - 1) and q + 1 has a same-key candidate
       if (LZ && l >= a.m && l < min(a.M, n - q - 1) && ((S.cand[(q + 1) >> 5] >> ((q + 1) & 31u)) & 1u)) {
-        cr = best_match(S, q + 1, n, nruns, a, lane, l);  // exact if > l
+        cr = best_match<BIG>(S, q + 1, n, nruns, a, lane, l);  // exact if > l
         cq = q + 1;
         if ((cr >> 16) > l) l = 0;  // deferred: x[q] is a literal
       }
@@ -366,8 +400,8 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     {
       const uint32_t w = p >> 5, sh = p & 31u;
       const uint32_t mask = cnt >= 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
-      red_or_if(lane == 0, &tbk[w], mask << sh);
-      red_or_if(lane == 0 && sh + cnt > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
+      tb_or_if<BIG>(lane == 0, &tbk[w], mask << sh);
+      tb_or_if<BIG>(lane == 0 && sh + cnt > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
       st_u16_if(lane == 0 && tok_len > 1, d1 + q, 0xFFFFu - (r & 0xFFFFu));  // d - 1
     }
     // does this stretch meet the successor's parse?
@@ -508,7 +542,9 @@ template <int K, bool G1 = false>
 struct MaxThreads {
   static constexpr int value =
       G1 ? 32 * K
-         : (K == 1 ? 320 : (K == 2 ? 640 : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : LZR_K8_THREADS))));
+         : (K == 1 ? 320
+                   : (K == 2 ? 640
+                             : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : (K == 16 ? 512 : LZR_K8_THREADS)))));
 };
 template <int K, bool G1 = false>
 struct MinBlocks {
@@ -519,7 +555,7 @@ struct MinBlocks {
 #endif
 constexpr uint32_t kG1MaxWaves = LZR_G1_MAX_WAVES;  // launches of fewer chunk waves than this use G1
 
-template <int K, int NS, bool LZ, bool G1>
+template <int K, int NS, bool LZ, bool G1, bool BIG>
 __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::value)
     lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
@@ -536,17 +572,20 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
   uint32_t* bms = reinterpret_cast<uint32_t*>(base + a.L.off_bm);
   S.cand = bms;
   S.cb = bms + nw;
-  S.tb = bms + 2 * nw;
-  S.runs = S.tb + K * a.L.tb_words;
+  S.tb = bms + 2 * nw;  // (big chunks: in the global scratch, below)
+  S.runs = BIG ? bms + 2 * nw : S.tb + K * a.L.tb_words;
   S.ctrl = S.runs + a.L.max_runs;
   S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
   const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;  // NS == a.L.nsplit
   const uint32_t lt = lanemask_lt();
   const uint32_t tid = k * 32 + lane;
-  // (d-1) of recorded matches: a per-group global scratch reused chunk after
-  // chunk (stays in L2); read back only at the final match starts
-  uint16_t* d1 = reinterpret_cast<uint16_t*>(
-      a.scratch + ((size_t)blockIdx.x * (blockDim.x / (32 * K)) + g) * (2 * (size_t)a.C));
+  // per-group global scratch, reused chunk after chunk (stays in L2): (d-1) of
+  // recorded matches, read back only at the final match starts; big chunks:
+  // then the K token-start bitmaps
+  uint8_t* gscr = a.scratch + ((size_t)blockIdx.x * (blockDim.x / (32 * K)) + g) *
+                                 (BIG ? enc_scratch_per_group(a.L, a.C) : 2 * (size_t)a.C);
+  uint16_t* d1 = reinterpret_cast<uint16_t*>(gscr);
+  if (BIG) S.tb = reinterpret_cast<uint32_t*>(gscr + 2 * (size_t)a.C);
 
   if (k == 0 && lane == 0) {
     mbar_init(S.bar, 1);
@@ -679,7 +718,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     // before it -- instead of warp 0 alone while the others wait at the barrier
     // (greedy only: in the lazy kernel the same change measured 38.5 -> 35.9
     // GB/s mix -- a different register allocation of its longer walk)
-    constexpr bool kParScan = LZR_PAR_SCAN && (K == 4 || (K == 8 && LZR_PAR_SCAN8)) && NS + 2 <= K && !LZ;
+    constexpr bool kParScan = LZR_PAR_SCAN && (K == 4 || (K >= 8 && LZR_PAR_SCAN8)) && NS + 2 <= K && !LZ;
     if (kParScan && (B / 2) % (32 * K) == 0) {
       const uint32_t q0 = k * (B / 2 / K), q1 = q0 + B / 2 / K;
       uint32_t carry = 0;
@@ -826,14 +865,14 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
       }
       for (uint32_t j = lane; j < min(nruns, a.L.max_runs); j += 32) {
         const uint32_t st = S.runs[j];
-        S.runs[j] = ((st + run_len(S.cb, st, n - st)) << 16) | st;
+        S.runs[j] = ((st + run_len(S.cb, st, n - st) - 1u) << 16) | st;  // (end - 1, start): 16 bits each
       }
     }
     GSYNC(4);
 
     // ---- mark the first entry of every non-empty bucket (the last split's
     //      cursor of h = end of h)
-    {
+    if (!BIG) {  // (big chunks: bucket ends instead of marks)
       const uint16_t* endc = S.slot + (NS - 1) * B;
       for (uint32_t hh = tid; hh < B; hh += nthr) {
         const uint32_t st = hh ? endc[hh - 1] : 0u;
@@ -845,7 +884,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
     // ---- slot of each position and the candidate bitmap: the nearest same-key
     //      earlier position is the nearest same-key entry below in the bucket
     const uint32_t nidx = S.ctrl[kCtrlIdx];
-    for (uint32_t sl = tid; sl < nidx; sl += nthr) {
+    for (uint32_t sl = tid; sl < nidx && !BIG; sl += nthr) {
       const uint32_t e = S.sorted[sl];
       const uint32_t q = e & kPos;
       S.slot[q] = (uint16_t)sl;
@@ -863,6 +902,22 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         }
         if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
       }
+    }
+    for (uint32_t sl = tid; sl < nidx && BIG; sl += nthr) {
+      // big chunks: the bucket's first entry from the bucket ends
+      const uint32_t q = S.sorted[sl];
+      const uint32_t kq = ld32u(S.data, q) & a.kmask;
+      const uint32_t h = khash(kq, hb, a.kmask);
+      const uint32_t bs = h ? S.slot[h - 1] : 0u;
+      bool has = false;
+      for (uint32_t s2 = sl; s2 > bs;) {
+        const uint32_t q2 = S.sorted[--s2];
+        if ((ld32u(S.data, q2) & a.kmask) == kq) {
+          has = q - q2 <= a.W;
+          break;
+        }
+      }
+      if (has) atomicOr(&S.cand[q >> 5], 1u << (q & 31u));
     }
     if (skipr && nruns) {
       // not-indexed positions (key = k copies of one byte): inside a run (the
@@ -912,7 +967,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         nb = walk_bound(n, k + 1, K);
       }
       if (start < n && (k == 0 || start > 0))
-        walk_segment<K, LZ>(S, d1, k, start, nb, n, P, nruns, a, lane);
+        walk_segment<K, LZ, BIG>(S, d1, k, start, nb, n, P, nruns, a, lane);
     }
     GSYNC(7);
 
@@ -1026,7 +1081,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
             const uint32_t j = tbase + __popc(t & ((1u << bit) - 1u));
             atomicOr(&S.cb[j >> 5], 1u << (j & 31u));
             const uint32_t pm = (w << 5) + bit;
-            S.slot[pm] = __ldcg(d1 + pm);  // the slot array is dead after the walk
+            if (!BIG) S.slot[pm] = __ldcg(d1 + pm);  // the slot array is dead after the walk
           }
         } else {
           const uint32_t nwr = min(32u, w_hi - w0);
@@ -1045,7 +1100,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
                 uint32_t b = S.cand[ww] & (0xFFFFFFFFu << ((p + 1) & 31u));
                 while (!b) b = S.cand[++ww];
                 const uint32_t l = (ww << 5) + (uint32_t)(__ffs(b) - 1) - p;
-                const uint32_t dm1 = S.slot[p];
+                const uint32_t dm1 = BIG ? (uint32_t)__ldcg(d1 + p) : (uint32_t)S.slot[p];
                 ob[pos] = (uint8_t)(dm1 & 0xFF);
                 ob[pos + 1] = (uint8_t)(dm1 >> 8);
                 ob[pos + 2] = (uint8_t)(l - a.m);
@@ -1070,7 +1125,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
   }
 }
 
-template <int K, int NS, bool LZ, bool G1 = false>
+template <int K, int NS, bool LZ, bool G1 = false, bool BIG = false>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
   const int max_groups = MaxThreads<K, G1>::value / (32 * K);
@@ -1098,7 +1153,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   {
     std::lock_guard<std::mutex> lk(mu);
     if (!cache[dev].attr) {
-      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1>,
+      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1, BIG>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
       if (err != cudaSuccess) return err;
       cache[dev].attr = true;
@@ -1109,7 +1164,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
     // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
     if (MinBlocks<K, G1>::value > 1 &&
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1>,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG>,
                                                       groups * 32 * K, smem) != cudaSuccess)
       per_sm = 1;
     if (per_sm < 1) per_sm = 1;
@@ -1120,7 +1175,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
-  lzr_encode_kernel<K, NS, LZ, G1><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS, LZ, G1, BIG><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -1153,6 +1208,9 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
         case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;
       }
+    case 16:  // big chunks (C > 32 KiB): one group of 16 warps per SM
+      if (!enc_big(a.C) || a.L.nsplit != 1) return cudaErrorInvalidConfiguration;
+      return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);
     case 8:
       switch (a.L.nsplit) {
         case 1: return launch_k<8, 1, LZ>(a, sm_count, smem_optin, s, launches);

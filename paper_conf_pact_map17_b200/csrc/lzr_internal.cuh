@@ -94,7 +94,19 @@ __host__ __device__ inline uint32_t enc_max_runs(uint32_t C) {
 
 struct EncLayout {
   uint32_t K, nsplit, max_runs, off_sorted, off_slot, off_bm, off_mbar, per_group, hbits, bm_words, tb_words, fbits;
+  // (no further fields: the kernels take EncArgs by value, and ptxas's register
+  // allocation of the 4 KiB kernel was measured to change -- a spill -- with its size)
 };
+
+// Chunks above 32 KiB (up to the format's 64 KiB): one
+// chunk's index no longer fits next to 15-bit positions and per-position slot
+// arrays, so the big layout keeps full 16-bit positions in the index, bucket
+// ends instead of bucket-start marks (B = 8192 buckets), no per-position slot
+// array (a search finds p's own entry inside its bucket), and the K
+// token-start bitmaps of the walk segments in the group's global scratch
+// (L2-resident, next to the (d-1) scratch).
+constexpr uint32_t kBigChunk = 32768;
+constexpr uint32_t kBigHashBits = 13;
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
   uint32_t hb = 0;
@@ -105,12 +117,15 @@ __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
 // K warps per chunk; NS of them share the index scatter, each with its own
 // cursor array, so NS * B u16 counters must fit the 2 max(C, B)-byte slot
 // region: B = (largest power of two <= C) / NS
+__host__ __device__ inline bool enc_big(uint32_t C) { return C > kBigChunk; }
+
 __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t NS) {
   EncLayout L;
   L.K = K;
-  L.hbits = enc_hash_bits(C);
+  const bool big = enc_big(C);
+  L.hbits = big ? kBigHashBits : enc_hash_bits(C);
   L.nsplit = 1;
-  while (L.nsplit < NS && L.hbits > 4) {
+  while (!big && L.nsplit < NS && L.hbits > 4) {
     --L.hbits;
     L.nsplit <<= 1;
   }
@@ -122,18 +137,26 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
   L.off_sorted = o;
   o += 2 * C;  // u16 positions grouped by hash bucket, ascending
   L.off_slot = o;
-  o += 2 * (C > B ? C : B);  // u16 histogram -> cursors -> slot of each position
+  // u16 histogram -> cursors -> slot of each position (big: -> bucket ends)
+  o += big ? 2 * B : 2 * (C > B ? C : B);
   L.off_bm = o;
   L.bm_words = (C + 31) / 32 + 1;  // candidate / byte-change: +1 for two-word funnel reads
   L.tb_words = (C + 31) / 32;      // per-segment token-start bitmaps
-  // candidate, byte-change, K token-start bitmaps; run list; ctrl (4 + 2K words)
+  // candidate, byte-change, K token-start bitmaps (big: in global scratch); run
+  // list; ctrl (4 + 2K words)
   L.max_runs = enc_max_runs(C);
-  o += 4 * (2 * L.bm_words + K * L.tb_words + L.max_runs + 4 + 2 * K);
+  o += 4 * (2 * L.bm_words + (big ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K);
   o = align_up(o, 8);
   L.off_mbar = o;
   o += 8;
   L.per_group = align_up(o, 16);  // next group's chunk buffer: 16-byte aligned (TMA)
   return L;
+}
+
+// global scratch bytes per resident group: (d-1) per position (u16), + the K
+// token-start bitmaps when big
+__host__ __device__ inline size_t enc_scratch_per_group(const EncLayout& L, uint32_t C) {
+  return enc_big(C) ? align_up_z(2 * (size_t)C + 4 * (size_t)L.K * L.tb_words, 256) : 2 * (size_t)C;
 }
 
 struct EncArgs {
@@ -154,7 +177,8 @@ struct EncArgs {
 struct WsLayout {
   size_t ctrl_off, slots_off, scratch_off, scan_off, total;
 };
-constexpr uint32_t kMaxGroupsPerSm = 16;  // scratch bound: groups per CTA (one CTA per SM)
+constexpr uint32_t kMaxGroupsPerSm = 16;  // scratch bound: resident groups per SM
+constexpr uint32_t kSmemPerSm = 233472;   // shared memory per SM (228 KB)
 size_t scan_ws_bytes(size_t n);
 WsLayout ws_layout(size_t n_bytes, const lzr_params* p);
 

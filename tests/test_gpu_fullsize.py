@@ -75,7 +75,7 @@ def _sampled_check(lzr, ref, xd, C, every, roundtrip=True, full=True):
     del out
 
 
-@pytest.mark.parametrize("C", [4096, 8192, 16384, 32768])
+@pytest.mark.parametrize("C", [4096, 8192, 16384, 32768, 65536])
 def test_config3_1gib_sampled(lzr, ref, C):
     xd = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
     synth.fill_device(xd, C, "mix")

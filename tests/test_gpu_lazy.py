@@ -37,6 +37,7 @@ def test_lazy_adversarial_bitexact(lzr, ref, name, x):
     (4096, 4096, 3, 258), (4096, 4096, 5, 40), (4096, 4096, 3, 3), (4096, 4096, 4, 5),
     (4096, 1000, 4, 259), (4096, 1, 4, 259), (4096, 33, 6, 261), (16, 16, 3, 258), (528, 300, 4, 20),
     (8192, 8192, 4, 259), (8192, 2048, 4, 259), (16384, 16384, 4, 259), (32768, 32768, 4, 259),
+    (65536, 65536, 4, 259), (65536, 30000, 3, 200),
 ])
 def test_lazy_param_grid_bitexact(lzr, ref, C, W, m, M):
     n = max(C * 3 + C // 3 + 1, 3000)

@@ -111,6 +111,10 @@ def test_adversarial_bitexact(lzr, ref, name, x):
     (4096, 1000, 4, 259), (4096, 1, 4, 259), (4096, 2, 3, 100), (4096, 33, 6, 261),
     (16, 16, 3, 258), (16, 5, 4, 259), (48, 48, 4, 259), (528, 300, 4, 20),
     (8192, 8192, 4, 259), (16384, 16384, 4, 259), (32768, 32768, 4, 259),
+    # big chunks (C > 32 KiB): 16-bit positions, bucket ends,
+    # in-bucket search for p's entry, walk bitmaps in global scratch
+    (65536, 65536, 4, 259), (65536, 65536, 3, 258), (65536, 20000, 4, 259), (40000, 40000, 4, 259),
+    (32784, 32784, 5, 100),
 ])
 def test_param_grid_bitexact(lzr, ref, C, W, m, M):
     p = lzr.Params(chunk_size=C, window=W, min_match=m, max_match=M)
@@ -322,7 +326,8 @@ def test_gpu_decoder_fuzz_vs_oracle(lzr, ref, C, m, cls):
 
 
 @pytest.mark.parametrize("C,W,m", [(4096, 4096, 3), (4096, 4096, 5), (8192, 8192, 4), (32768, 32768, 4),
-                                   (4096, 4095, 4), (4096, 4094, 4), (8192, 8192, 3)])
+                                   (4096, 4095, 4), (4096, 4094, 4), (8192, 8192, 3),
+                                   (65536, 65536, 4), (65536, 65536, 3), (65536, 65535, 4)])
 def test_runs_structures_param_grid(lzr, ref, C, W, m):
     """Run-heavy chunks across m, C and W around the 'every prefix in the window'
     boundary: the index leaves repeated-byte keys out (run-aware search only) iff
@@ -405,3 +410,23 @@ def test_other_stream_dedup_and_compress(lzr, ref):
         r_out, _, _, r_tot = ref.compress(ub, ref.Params())
         assert int(res["total"].item()) == r_tot
         assert np.array_equal(res["out"][:r_tot].cpu().numpy(), r_out)
+
+
+@pytest.mark.parametrize("cls", ["text", "zeroruns", "random", "cr2"])
+def test_big_chunk_classes_bitexact(lzr, ref, cls):
+    """C = W = 64 KiB (the format's largest window, d - 1 < 2^16) on every class,
+    plus a whole-chunk zero run (run end = 65536) and a period-3 chunk."""
+    C = 65536
+    x = synth.fill_host(C * 3 + 4112, C, cls, seed=64)
+    _check_full(lzr, ref, x, lzr.Params(chunk_size=C))
+
+
+def test_big_chunk_edge_inputs(lzr, ref):
+    C = 65536
+    _check_full(lzr, ref, np.zeros(C * 2, np.uint8), lzr.Params(chunk_size=C))
+    per = np.tile(np.frombuffer(b"xyz", np.uint8), C // 3 + 1)[: C + 77].copy()
+    _check_full(lzr, ref, per, lzr.Params(chunk_size=C))
+    rng = np.random.default_rng(9)
+    words = [bytes(rng.integers(97, 123, int(rng.integers(3, 9)), dtype=np.uint8)) for _ in range(40)]
+    t = b" ".join(words[int(i)] for i in rng.integers(0, 40, 30000))[: C * 2 - 5]
+    _check_full(lzr, ref, np.frombuffer(t, np.uint8).copy(), lzr.Params(chunk_size=C))

@@ -68,7 +68,7 @@ def _const_closed_form(n, m, M):
     return min(S, n) if S < n else n
 
 
-@pytest.mark.parametrize("n,expect", [(4096, 52), (8192, 102), (16384, 202), (32768, 398)])
+@pytest.mark.parametrize("n,expect", [(4096, 52), (8192, 102), (16384, 202), (32768, 398), (65536, 795)])
 def test_constant_chunk_sizes(ref, n, expect):
     p = ref.Params(chunk_size=n)
     s = ref.compress_chunk(bytes(n), p)
