@@ -536,6 +536,8 @@ def run_dedup(a):
                                 "sample": f"first {smp >> 20} MiB of the logical stream: SHA-1, "
                                           f"index, compress of its {ub.size >> 20} MiB unique, {dt:.1f} s",
                                 "index_parity_vs_gpu": "bit-exact" if ok else "MISMATCH"}
+    if world == 1 and not a.no_cpu:
+        line["integration"] = integration_options(lzr, p, dev)
     if grank == 0:
         print(json.dumps(line), flush=True)
     R.close()
@@ -573,6 +575,32 @@ def per_class(lzr, synth, p, n, dev, stream, steps=5, warmup=2):
                     "round_trip": "ok" if ok else "MISMATCH"}
     del x, ws, y
     return res
+
+
+def integration_options(lzr, p, dev, dummy_bytes=64 << 20):
+    """SURVEY.md §8(f) N3 / PAPER.md P:20 §4(3): the integration options --
+    dedup and compression each on the GPU or the CPU, or the compression split
+    between both -- timed end to end from host memory on a dummy dedup-2.0
+    stream ("compared using dummy I/O to determine the best fit for
+    throughput"); the fastest is the pick.  The CPU arm is cpuref (hash-chain
+    compressor, thread per chunk) + hashlib SHA-1 dedup on all host cores."""
+    import cpuref
+    import synth
+    from paper_conf_pact_map17_b200.integration import CpuArm, Integrated
+
+    cores = len(os.sched_getaffinity(0))
+    arm = CpuArm(compress=lambda x, q: cpuref.compress(x, cpuref.Params(chunk_size=q.chunk_size, window=q.window,
+                                                                         parse=q.parse), n_threads=cores),
+                 dedup=lambda x, C: cpuref.dedup(x, C, cores), cores=cores)
+    it = Integrated(p, arm, dev)
+    dummy = synth.fill_host(dummy_bytes, p.chunk_size, "mix_dedup", seed=0xD0)
+    cal = it.calibrate(dummy, repeats=2)
+    return {"gbs_logical": {k: round(v, 3) for k, v in cal["gbs"].items()}, "pick": cal["pick"],
+            "split_fraction_cpu": round(cal["split_fraction"], 4), "cpu_cores": cores,
+            "dummy": f"{dummy_bytes >> 20} MiB dedup-2.0 mix stream, host memory in and out "
+                     "(H2D/D2H inside the GPU placements), best of 2",
+            "paper": "P:20 §4(3): GPU for both / one / none, compared by dummy I/O; the paper's pick: "
+                     "'Allocating the GPU for compression is the best choice'"}
 
 
 def main():

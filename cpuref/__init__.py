@@ -1,12 +1,15 @@
-"""Fast exact CPU compressor -- TEST INFRASTRUCTURE AND CPU BASELINE ONLY
-(``cpuref/lzr_fast.c``).
+"""Fast exact CPU compressor -- the paper's CPU arm, TEST INFRASTRUCTURE AND
+CPU BASELINE (``cpuref/lzr_fast.c``).
 
 The same result as the plain oracle (``oracle/``), found with hash chains and
 a run-aware search instead of an exhaustive scan, multi-threaded per chunk
 (§3.2(1)).  Pinned to the oracle by ``tests/test_cpuref.py``.  Used for
-whole-stream GPU parity at multi-GiB sizes and as the CPU arm of the paper's
-GPU-usage decision (§3.2(3)) in ``bench.py``.  Only ``tests/``,
+whole-stream GPU parity at multi-GiB sizes, as the CPU arm of the paper's
+GPU-usage decision (§3.2(3)) in ``bench.py``, and injected by bench.py /
+the tests as the CPU side of the integration-option selection
+(``paper_conf_pact_map17_b200.integration``, §4(3)).  Only ``tests/``,
 ``bench.py`` and ``tools/`` import it; the product package never does.
+``dedup`` is the CPU dedup arm (hashlib SHA-1 + a first-occurrence dict, R17/R18).
 """
 from __future__ import annotations
 
@@ -92,3 +95,31 @@ def compress(x, p: Params, n_threads: int | None = None, slots: np.ndarray | Non
     if st != 0:
         raise ValueError(f"lzr_fast_compress status {st}")
     return buf[: tot.value], sizes[:N], offs[:N], tot.value
+
+
+def dedup(x, chunk_size: int, n_threads: int | None = None):
+    """CPU dedup arm: SHA-1 of every chunk (hashlib, threads; a short tail chunk
+    hashes its own length, R17), then first-occurrence indexing in stream order
+    (R18).  -> (index int64[N], unique int32[N])."""
+    import hashlib
+    from concurrent.futures import ThreadPoolExecutor
+
+    a = np.ascontiguousarray(x, dtype=np.uint8).reshape(-1)
+    C = chunk_size
+    N = -(-a.size // C)
+    mv = memoryview(a)
+    if n_threads is None:
+        n_threads = len(os.sched_getaffinity(0))
+    step = max(1, -(-N // (4 * n_threads)))
+
+    def part(lo):
+        return [hashlib.sha1(mv[i * C: min(a.size, (i + 1) * C)]).digest() for i in range(lo, min(N, lo + step))]
+
+    with ThreadPoolExecutor(n_threads) as ex:
+        fps = [d for blk in ex.map(part, range(0, N, step)) for d in blk]
+    first = {}
+    index = np.empty(N, np.int64)
+    for i, d in enumerate(fps):
+        index[i] = first.setdefault(d, i)
+    unique = (index == np.arange(N)).astype(np.int32)
+    return index, unique

@@ -242,10 +242,15 @@ __device__ __forceinline__ uint32_t best_match_runs(const Smem& S, uint32_t p, u
 // the generic path then evaluates only candidates that also match the byte at
 // offset floor; the result is exact whenever it exceeds floor (every candidate
 // reaching the maximum passes that test), otherwise it is some value <= floor.
+// prevb <= 0xFF (lazy parse, p = q0 + 1 after a match of length floor < cap at
+// q0, prevb = x[q0]): a candidate r preceded by prevb (x[r-1] == x[q0]) is
+// skipped -- r - 1 then has q0's key at the same distance, so it is a
+// candidate of q0, whose best length floor is below q0's cap; hence
+// LCP(q0, r-1) <= floor and LCP(p, r) = LCP(q0, r-1) - 1 < floor.
 template <bool BIG>
 __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32_t n,
                                                uint32_t nruns, const EncArgs& a, uint32_t lane,
-                                               uint32_t floor = 0) {
+                                               uint32_t floor = 0, uint32_t prevb = 0x100u) {
   const uint8_t* data = S.data;
   const uint32_t cap = min(a.M, n - p);  // p < n - m + 1  =>  cap >= m >= k
   const uint32_t kp = ld32u(data, p) & a.kmask;
@@ -309,7 +314,8 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
     if (m_first) lim = (uint32_t)__ffs(m_first);
     if (m_stop) lim = min(lim, (uint32_t)(__ffs(m_stop) - 1));
     uint32_t pk = 0;
-    if (lane < lim && (blen == 0 || data[q + blen] == data[p + blen])) {
+    if (lane < lim && (blen == 0 || data[q + blen] == data[p + blen]) &&
+        (prevb > 0xFFu || q == 0 || data[q - 1] != prevb)) {
       uint32_t l;
       if (rp) {
         if ((ld32u(data, q) & a.kmask) != kp) {
@@ -389,7 +395,7 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       // LZ: a longer match at q + 1 is possible only if l is below its cap
       // min(M, n - q - 1) and q + 1 has a same-key candidate
       if (LZ && l >= a.m && l < min(a.M, n - q - 1) && ((S.cand[(q + 1) >> 5] >> ((q + 1) & 31u)) & 1u)) {
-        cr = best_match<BIG>(S, q + 1, n, nruns, a, lane, l);  // exact if > l
+        cr = best_match<BIG>(S, q + 1, n, nruns, a, lane, l, S.data[q]);  // exact if > l
         cq = q + 1;
         if ((cr >> 16) > l) l = 0;  // deferred: x[q] is a literal
       }

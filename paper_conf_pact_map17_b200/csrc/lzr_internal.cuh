@@ -105,7 +105,10 @@ struct EncLayout {
 // array (a search finds p's own entry inside its bucket), and the K
 // token-start bitmaps of the walk segments in the group's global scratch
 // (L2-resident, next to the (d-1) scratch).
-constexpr uint32_t kBigChunk = 32768;
+#ifndef LZR_BIG_CHUNK
+#define LZR_BIG_CHUNK 32768
+#endif
+constexpr uint32_t kBigChunk = LZR_BIG_CHUNK;
 constexpr uint32_t kBigHashBits = 13;
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {

@@ -86,3 +86,17 @@ def test_validation():
     assert cpuref.validate(cpuref.Params(parse=2)) == -2
     assert cpuref.validate(cpuref.Params(tie_break=1)) == -2
     assert cpuref.validate(cpuref.Params(chunk_size=24)) == -1
+
+
+def test_cpu_dedup_arm_equals_oracle_index(ref):
+    """The CPU dedup arm of the integration options (hashlib SHA-1 + first
+    occurrence) == the oracle's fingerprints + index (R17, R18), tail chunk included."""
+    import cpuref
+    import synth
+
+    for n, C in [((1 << 20) + 777, 4096), (300 * 512, 512), (5, 4096)]:
+        x = synth.fill_host(n, C, "mix_dedup", seed=n)
+        idx, un = cpuref.dedup(x, C, 4)
+        r_idx, r_hit, _ = ref.dedup_index(ref.fingerprints(x, C), 0)
+        assert np.array_equal(idx.astype(np.uint64), r_idx)
+        assert np.array_equal(un.astype(bool), r_hit == 0)
