@@ -28,14 +28,18 @@ def deps():
         os.path.join(ROOT, "include", "lzr.h")]
 
 
-def source_hash() -> str:
-    """Hash of the kernel sources (csrc + include/lzr.h) that liblzr.so is built
-    from: stamps ncu captures so that the bench drops profile-derived keys
-    taken on a different build (no toolchain needed to compute it)."""
+def source_hash(kernel: str = "encode") -> str:
+    """Hash of the sources one kernel of liblzr.so is built from (encode.cu +
+    the shared header + include/lzr.h for "encode"; every source for "all"):
+    stamps ncu captures so that the bench drops profile-derived keys taken on
+    a different build of that kernel (no toolchain needed to compute it)."""
     import hashlib
 
+    files = deps() if kernel == "all" else [
+        os.path.join(CSRC, f"{kernel}.cu"), os.path.join(CSRC, "lzr_internal.cuh"),
+        os.path.join(ROOT, "include", "lzr.h")]
     h = hashlib.sha256()
-    for d in deps():
+    for d in files:
         h.update(os.path.basename(d).encode())
         with open(d, "rb") as f:
             h.update(f.read())
