@@ -4,8 +4,9 @@
 // The four flag bytes of a step are a short dependent chain (group g + 1
 // starts 9 + 2 popc(f_g) bytes after group g); then lane t owns token t: its
 // stream offset is ip_g + 1 + j + 2 popc(f_g below j), its output position a
-// 32-lane prefix sum of token lengths.  Token headers are read straight from
-// global memory (L1-cached byte loads, never outside [src, src + S)).  The chunk
+// 32-lane prefix sum of token lengths.  A step's stream bytes come from a
+// 128-byte window held one word per lane (loaded coalesced while the previous
+// step copies, bytes outside [src, src + S) read as 0) by shuffle.  The chunk
 // is rebuilt in shared memory: literals of the step are stored in parallel,
 // then the step's matches are resolved in rounds -- a match whose source bytes
 // lie below the first unresolved match's output (or that is the first one) is
@@ -31,6 +32,14 @@ namespace lzr {
 namespace {
 
 constexpr int kDecWarpsMax = 16;
+// CTA shape of the decode grid (see launch_decode): 2 warps, and enough
+// resident CTAs per SM that registers do not cut occupancy below ~48 warps
+#ifndef LZR_DEC_WARPS
+#define LZR_DEC_WARPS 2
+#endif
+#ifndef LZR_DEC_MINB
+#define LZR_DEC_MINB 24
+#endif
 constexpr int32_t kNoError = 0x7F7F7F7F;
 constexpr uint32_t kLaneCopyMax = 16;  // matches up to this length: one lane, byte-serial
 // (measured and not kept, 1 x B200, 256 MiB, output GB/s mix/text/zero-runs:
@@ -52,12 +61,8 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
   return v;
 }
 
-// stream byte x, 0 past the end (the caller flags the error)
-__device__ __forceinline__ uint32_t sbyte(const uint8_t* src, uint32_t S, uint32_t x) {
-  return x < S ? (uint32_t)__ldg(src + x) : 0u;
-}
 
-__global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
+__global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_kernel(
     const uint8_t* __restrict__ comp, const uint32_t* __restrict__ sizes,
     const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C, uint32_t m,
     uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride) {
@@ -91,18 +96,29 @@ __global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
       continue;
     }
     bool bad = S > n;
+    // A step reads at most 4 groups (<= 100 bytes) from ip.  The 128 stream
+    // bytes from ip (32 aligned words, one per lane: a coalesced load, bytes
+    // outside the stream read as 0) are loaded before the step -- the next
+    // step's window is issued as soon as this step's end is known, so its
+    // latency hides under the match copies -- and the parse takes its bytes
+    // from the window by shuffle instead of a chain of dependent loads.
+    const uint32_t mis = (uint32_t)((uintptr_t)src & 3u);
     uint32_t ip = 0, op = 0;
+    uint32_t wbase = mis >> 2;  // first word of the window (aligned view src - mis)
+    uint32_t win = bad ? 0u : load_word(src, mis, S, wbase + lane);
     while (!bad && op < n) {
-      // a step reads at most 4 groups (<= 100 bytes) from ip: away from the
-      // stream's end no read needs its bounds check
-      const bool safe = ip + 100 <= S;
+      const uint32_t wb = wbase, wv = win;
+      auto sb = [&](uint32_t x) -> uint32_t {  // stream byte x (x <= ip + 101), 0 past the end
+        const uint32_t xx = x + mis;
+        return (__shfl_sync(kFull, wv, (xx >> 2) - wb) >> ((xx & 3u) << 3)) & 0xFFu;
+      };
       // the four groups of this step: flag byte and stream offset
       uint32_t f = 0, ipg = 0;
       {
         uint32_t x = ip;
 #pragma unroll
         for (uint32_t t = 0; t < 4; ++t) {
-          const uint32_t ft = safe ? (uint32_t)__ldg(src + x) : sbyte(src, S, x);
+          const uint32_t ft = sb(x);
           if (t == g) {
             f = ft;
             ipg = x;
@@ -113,11 +129,11 @@ __global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
       const uint32_t ism = (f >> j) & 1u;
       const uint32_t toff = ipg + 1u + j + 2u * __popc(f & below);
       const uint32_t tsz = 1u + 2u * ism;
-      const uint32_t b0 = safe ? (uint32_t)__ldg(src + toff) : sbyte(src, S, toff);
-      uint32_t b1 = 0, b2 = 0;
-      if (ism) {
-        b1 = safe ? (uint32_t)__ldg(src + toff + 1) : sbyte(src, S, toff + 1);
-        b2 = safe ? (uint32_t)__ldg(src + toff + 2) : sbyte(src, S, toff + 2);
+      const uint32_t b0 = sb(toff);
+      uint32_t b1 = sb(toff + 1), b2 = sb(toff + 2);  // (all lanes: shuffles)
+      if (!ism) {
+        b1 = 0;
+        b2 = 0;
       }
       const uint32_t tlen = ism ? b2 + m : 1u;
       const uint32_t d = (b0 | (b1 << 8)) + 1u;
@@ -146,6 +162,11 @@ __global__ void __launch_bounds__(32 * kDecWarpsMax) lzr_decode_kernel(
       }
       const uint32_t rmask = __ballot_sync(kFull, reached);  // a prefix of the lanes
       const uint32_t last = 31u - __clz(rmask);
+      {  // the next step's window, issued now
+        const uint32_t ipn = __shfl_sync(kFull, toff + tsz, last);
+        wbase = (ipn + mis) >> 2;
+        win = ipn < S ? load_word(src, mis, S, wbase + lane) : 0u;
+      }
       if (reached && !ism) obuf[ob] = (uint8_t)b0;
       __syncwarp();
       uint32_t pend = __ballot_sync(kFull, reached && ism);
@@ -216,9 +237,6 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
 // the end (1 x B200, 256 MiB, output GB/s mix/text/zero-runs: 16-warp one-wave
 // 290/214/596; full grids of 16/8/4/2/1-warp CTAs 302/309/347/380/369 mix,
 // text 239-242 except 211 at 1 warp (32 CTAs per SM = 32 warps))
-#ifndef LZR_DEC_WARPS
-#define LZR_DEC_WARPS 2
-#endif
 #ifndef LZR_DEC_ONEWAVE
 #define LZR_DEC_ONEWAVE 0
 #endif
