@@ -31,7 +31,6 @@ namespace lzr {
 
 namespace {
 
-constexpr int kDecWarpsMax = 16;
 // CTA shape of the decode grid (see launch_decode): 2 warps, and enough
 // resident CTAs per SM that registers do not cut occupancy below ~48 warps
 #ifndef LZR_DEC_WARPS
