@@ -12,6 +12,13 @@ for tool in memcheck racecheck synccheck initcheck; do
   timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 \
     python tools/prof_encode.py --cls mix --mib 2 --iters 1 --decode --chunk-size 8192 > $out/${tool}_mix8k.log 2>&1
   echo "$tool mix C=8192 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_mix8k.log | tail -1)"
+  # big chunks (C = 64 KiB: 16-bit index, L2 walk bitmaps) and the lazy parse
+  timeout 1200 compute-sanitizer --tool $tool --error-exitcode 9 \
+    python tools/prof_encode.py --cls mix --mib 4 --iters 1 --decode --chunk-size 65536 > $out/${tool}_mix64k.log 2>&1
+  echo "$tool mix C=65536 rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_mix64k.log | tail -1)"
+  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 \
+    python tools/prof_encode.py --cls mix --mib 2 --iters 1 --decode --parse 1 > $out/${tool}_lazy.log 2>&1
+  echo "$tool mix lazy rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_lazy.log | tail -1)"
   timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/prof_dedup.py > $out/${tool}_dedup.log 2>&1
   echo "$tool dedup rc=$? $(grep -E 'ERROR SUMMARY|RACECHECK SUMMARY|hazard' $out/${tool}_dedup.log | tail -1)"
 done
