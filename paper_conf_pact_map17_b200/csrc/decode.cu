@@ -128,11 +128,16 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       const uint32_t ism = (f >> j) & 1u;
       const uint32_t toff = ipg + 1u + j + 2u * __popc(f & below);
       const uint32_t tsz = 1u + 2u * ism;
-      const uint32_t b0 = sb(toff);
-      uint32_t b1 = sb(toff + 1), b2 = sb(toff + 2);  // (all lanes: shuffles)
-      if (!ism) {
-        b1 = 0;
-        b2 = 0;
+      // the token's 3 header bytes from the two window words around toff
+      uint32_t b0, b1, b2;
+      {
+        const uint32_t xx = toff + mis;
+        const uint32_t wi = (xx >> 2) - wb;
+        const uint32_t lo = __shfl_sync(kFull, wv, wi), hi = __shfl_sync(kFull, wv, wi + 1);
+        const uint32_t v = __funnelshift_r(lo, hi, (xx & 3u) << 3);
+        b0 = v & 0xFFu;
+        b1 = ism ? (v >> 8) & 0xFFu : 0u;
+        b2 = ism ? (v >> 16) & 0xFFu : 0u;
       }
       const uint32_t tlen = ism ? b2 + m : 1u;
       const uint32_t d = (b0 | (b1 << 8)) + 1u;
