@@ -174,6 +174,27 @@ def test_config2_full_size_sampled(lzr, ref):
     assert int(err.item()) == 0 and torch.equal(y, xd)
 
 
+def test_config2_full_size_every_chunk_vs_oracle(lzr, ref):
+    """All 65,536 chunks of the bench's 256 MiB mix stream vs the oracle itself
+    (thread per chunk on the host cores, ~20 s on 16): sizes, offsets, total
+    and every byte (full-size parity not only through cpuref)."""
+    import os
+
+    n = 256 << 20
+    p = lzr.Params()
+    xd = torch.empty(n, dtype=torch.uint8, device="cuda")
+    synth.fill_device(xd, 4096, "mix")
+    out, sizes, offs, total = lzr.compress(xd, p)
+    torch.cuda.synchronize()
+    tot = int(total.item())
+    r_out, r_sizes, r_offs, r_tot = ref.compress(xd.cpu().numpy(), _ref_params(ref, p),
+                                                 n_threads=len(os.sched_getaffinity(0)))
+    assert tot == r_tot
+    assert np.array_equal(sizes.cpu().numpy().view(np.uint32), r_sizes)
+    assert np.array_equal(offs.cpu().numpy().view(np.uint64), r_offs)
+    assert np.array_equal(out[:tot].cpu().numpy(), r_out)
+
+
 def test_cross_decode_with_oracle(lzr, ref):
     x = synth.fill_host(3 << 20, 4096, "cr2", seed=99)
     g_out, g_sizes, g_offs = _check_full(lzr, ref, x, lzr.Params(), roundtrip=False)
