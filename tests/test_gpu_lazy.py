@@ -66,3 +66,22 @@ def test_lazy_config2_full_size_sampled(lzr, ref):
     y, err = lzr.decompress(out, sizes, offs, n, p)
     torch.cuda.synchronize()
     assert int(err.item()) == 0 and torch.equal(y, xd)
+
+
+def test_lazy_config2_every_chunk_vs_oracle(lzr, ref):
+    """The lazy parse over all 65,536 chunks of the 256 MiB mix stream vs the
+    oracle itself (thread per chunk on the host cores), every byte."""
+    import os
+
+    n = 256 << 20
+    p = _lazy(lzr)
+    xd = torch.empty(n, dtype=torch.uint8, device="cuda")
+    synth.fill_device(xd, 4096, "mix")
+    out, sizes, offs, total = lzr.compress(xd, p)
+    torch.cuda.synchronize()
+    tot = int(total.item())
+    r_out, r_sizes, r_offs, r_tot = ref.compress(xd.cpu().numpy(), ref.Params(parse=1),
+                                                 n_threads=len(os.sched_getaffinity(0)))
+    assert tot == r_tot
+    assert np.array_equal(sizes.cpu().numpy().view(np.uint32), r_sizes)
+    assert np.array_equal(out[:tot].cpu().numpy(), r_out)
