@@ -44,9 +44,16 @@ cudaError_t dev_info(DevInfo* out) {
 
 bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
-// Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 above (fewer
-// chunks fit one SM's shared memory, so each gets more warps).
+// Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 up to 16 KiB
+// (fewer chunks fit one SM's shared memory, so each gets more warps), 16 above:
+// one chunk per SM, walk bitmaps in the L2 scratch (32 KiB mix 12.0 -> 17.4
+// GB/s, text 5.7 -> 8.5, zero-runs 30.5 -> 37.2; at 16 KiB 16 warps lose to
+// two groups of 8: 19.6 vs 25.9).
 // LZR_ENCODE_WARPS=1,2,3,4,8 overrides (tuning).
+// chunks above this size get 16 warps (walk bitmaps in the L2 scratch)
+#ifndef LZR_K16_MIN
+#define LZR_K16_MIN 16384
+#endif
 uint32_t enc_warps_per_chunk(uint32_t C) {
   static int env = -1;
   if (env < 0) {
@@ -55,12 +62,12 @@ uint32_t enc_warps_per_chunk(uint32_t C) {
   }
   if (C > kBigChunk) return 16u;  // the big-chunk layout (lzr_internal.cuh) is built for 16
   if (env > 0) return (uint32_t)env;
-  return C > 4096 ? 8u : (C >= 1024 ? 4u : 1u);
+  return C > LZR_K16_MIN ? 16u : (C > 4096 ? 8u : (C >= 1024 ? 4u : 1u));
 }
 
 // warps that share the index scatter (each a contiguous position range with
 // its own cursor array; the hash table shrinks by the same factor)
-uint32_t enc_scatter_splits(uint32_t K) {
+uint32_t enc_scatter_splits(uint32_t K, uint32_t C) {
   static int env = -1;
   if (env < 0) {
     const char* e = getenv("LZR_ENCODE_SPLITS");
@@ -68,7 +75,7 @@ uint32_t enc_scatter_splits(uint32_t K) {
   }
   // default (config-3 sweep, 1 x B200): 1 split at K = 4 (C = 4 KiB: the full
   // C-bucket table matters more than the serial scatter), 4 at K = 8
-  if (K > 8) return 1u;  // big chunks: one scatter (their B counters fill the slot region)
+  if (K > 8) return C > kBigChunk ? 1u : 4u;  // big chunks: one scatter (B counters fill the slot region)
   const uint32_t ns = env > 0 ? (uint32_t)env : (K >= 8 ? 4u : 1u);
   return K < 4 ? 1u : (ns < K ? ns : K);  // (kernels are instantiated for these)
 }
@@ -86,7 +93,7 @@ WsLayout ws_layout(size_t n_bytes, const lzr_params* p) {
   // by 16 per SM; the launch uses at most ceil(N / groups) CTAs, i.e. at most
   // N + 15 groups
   const uint32_t K = enc_warps_per_chunk((uint32_t)C);
-  const EncLayout L = enc_layout((uint32_t)C, K, enc_scatter_splits(K));
+  const EncLayout L = enc_layout((uint32_t)C, K, enc_scatter_splits(K, (uint32_t)C));
   size_t per_sm = kSmemPerSm / L.per_group;
   if (per_sm > kMaxGroupsPerSm) per_sm = kMaxGroupsPerSm;
   if (per_sm < 1) per_sm = 1;
@@ -175,7 +182,7 @@ int lzr_compress_encode(const void* d_in, size_t n_bytes, const lzr_params* p, u
   a.kbytes = p->min_match < 4 ? p->min_match : 4;
   a.kmask = a.kbytes == 4 ? 0xFFFFFFFFu : ((1u << (8 * a.kbytes)) - 1u);
   const uint32_t K = enc_warps_per_chunk(p->chunk_size);
-  a.L = enc_layout(p->chunk_size, K, enc_scatter_splits(K));
+  a.L = enc_layout(p->chunk_size, K, enc_scatter_splits(K, p->chunk_size));
   // one chunk's index must fit one CTA's shared memory (C <= 32 KiB: 15-bit
   // positions + bucket-start marks; above: the big-chunk layout)
   if ((int)a.L.per_group > di.smem_optin) return LZR_ERR_UNSUPPORTED;

@@ -351,7 +351,7 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
 #ifndef LZR_PUB
 #define LZR_PUB 64  // progress published every LZR_PUB bytes of parse
 #endif
-template <int K, bool LZ, bool BIG>
+template <int K, bool LZ, bool BIG, bool TBG>
 __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32_t k, uint32_t start,
                                              uint32_t nb, uint32_t n, uint32_t P, uint32_t nruns,
                                              const EncArgs& a, uint32_t lane) {
@@ -406,8 +406,8 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
     {
       const uint32_t w = p >> 5, sh = p & 31u;
       const uint32_t mask = cnt >= 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
-      tb_or_if<BIG>(lane == 0, &tbk[w], mask << sh);
-      tb_or_if<BIG>(lane == 0 && sh + cnt > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
+      tb_or_if<TBG>(lane == 0, &tbk[w], mask << sh);
+      tb_or_if<TBG>(lane == 0 && sh + cnt > 32, &tbk[w + 1], sh ? mask >> (32 - sh) : 0u);
       st_u16_if(lane == 0 && tok_len > 1, d1 + q, 0xFFFFu - (r & 0xFFFFu));  // d - 1
     }
     // does this stretch meet the successor's parse?
@@ -579,7 +579,10 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
   S.cand = bms;
   S.cb = bms + nw;
   S.tb = bms + 2 * nw;  // (big chunks: in the global scratch, below)
-  S.runs = BIG ? bms + 2 * nw : S.tb + K * a.L.tb_words;
+  // token-start bitmaps of the walk segments in the global scratch: big chunks
+  // and the 16-warp groups of chunks above 16 KiB
+  constexpr bool TBG = BIG || K == 16;
+  S.runs = TBG ? bms + 2 * nw : S.tb + K * a.L.tb_words;
   S.ctrl = S.runs + a.L.max_runs;
   S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
   const uint32_t hb = a.L.hbits, B = 1u << hb, fb = a.L.fbits;  // NS == a.L.nsplit
@@ -589,9 +592,9 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
   // recorded matches, read back only at the final match starts; big chunks:
   // then the K token-start bitmaps
   uint8_t* gscr = a.scratch + ((size_t)blockIdx.x * (blockDim.x / (32 * K)) + g) *
-                                 (BIG ? enc_scratch_per_group(a.L, a.C) : 2 * (size_t)a.C);
+                                 (TBG ? enc_scratch_per_group(a.L, a.C) : 2 * (size_t)a.C);
   uint16_t* d1 = reinterpret_cast<uint16_t*>(gscr);
-  if (BIG) S.tb = reinterpret_cast<uint32_t*>(gscr + 2 * (size_t)a.C);
+  if (TBG) S.tb = reinterpret_cast<uint32_t*>(gscr + 2 * (size_t)a.C);
 
   if (k == 0 && lane == 0) {
     mbar_init(S.bar, 1);
@@ -973,7 +976,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::va
         nb = walk_bound(n, k + 1, K);
       }
       if (start < n && (k == 0 || start > 0))
-        walk_segment<K, LZ, BIG>(S, d1, k, start, nb, n, P, nruns, a, lane);
+        walk_segment<K, LZ, BIG, TBG>(S, d1, k, start, nb, n, P, nruns, a, lane);
     }
     GSYNC(7);
 
@@ -1214,9 +1217,13 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
         case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;
       }
-    case 16:  // big chunks (C > 32 KiB): one group of 16 warps per SM
-      if (!enc_big(a.C) || a.L.nsplit != 1) return cudaErrorInvalidConfiguration;
-      return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+    case 16:  // chunks above 16 KiB: one group of 16 warps per SM
+      if (enc_big(a.C)) {
+        if (a.L.nsplit != 1) return cudaErrorInvalidConfiguration;
+        return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+      }
+      if (a.L.nsplit != 4) return cudaErrorInvalidConfiguration;
+      return launch_k<16, 4, LZ, false, false>(a, sm_count, smem_optin, s, launches);
     case 8:
       switch (a.L.nsplit) {
         case 1: return launch_k<8, 1, LZ>(a, sm_count, smem_optin, s, launches);

@@ -148,7 +148,8 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
   // candidate, byte-change, K token-start bitmaps (big: in global scratch); run
   // list; ctrl (4 + 2K words)
   L.max_runs = enc_max_runs(C);
-  o += 4 * (2 * L.bm_words + (big ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K);
+  const bool tbg = big || K == 16;  // walk bitmaps in the global scratch
+  o += 4 * (2 * L.bm_words + (tbg ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K);
   o = align_up(o, 8);
   L.off_mbar = o;
   o += 8;
@@ -159,7 +160,8 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
 // global scratch bytes per resident group: (d-1) per position (u16), + the K
 // token-start bitmaps when big
 __host__ __device__ inline size_t enc_scratch_per_group(const EncLayout& L, uint32_t C) {
-  return enc_big(C) ? align_up_z(2 * (size_t)C + 4 * (size_t)L.K * L.tb_words, 256) : 2 * (size_t)C;
+  return (enc_big(C) || L.K == 16) ? align_up_z(2 * (size_t)C + 4 * (size_t)L.K * L.tb_words, 256)
+                                   : 2 * (size_t)C;
 }
 
 struct EncArgs {
