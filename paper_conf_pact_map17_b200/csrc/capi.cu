@@ -44,15 +44,16 @@ cudaError_t dev_info(DevInfo* out) {
 
 bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
-// Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 up to 16 KiB
-// (fewer chunks fit one SM's shared memory, so each gets more warps), 16 above:
-// one chunk per SM, walk bitmaps in the L2 scratch (32 KiB mix 12.0 -> 17.4
-// GB/s, text 5.7 -> 8.5, zero-runs 30.5 -> 37.2; at 16 KiB 16 warps lose to
-// two groups of 8: 19.6 vs 25.9).
+// Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 up to 8 KiB
+// (fewer chunks fit one SM's shared memory, so each gets more warps), 16 above
+// with the walk bitmaps in the L2 scratch and <= 56 registers, so two 16 KiB
+// chunks (or one 32 KiB chunk) of 16 warps run per SM (1 x B200, 1 GiB mix,
+// GB/s: 16 KiB 25.9 -> 33.7, 32 KiB 12.0 -> 17.8; at 8 KiB 16 warps lose to
+// four groups of 8: 34.1 vs 44.0).
 // LZR_ENCODE_WARPS=1,2,3,4,8 overrides (tuning).
 // chunks above this size get 16 warps (walk bitmaps in the L2 scratch)
 #ifndef LZR_K16_MIN
-#define LZR_K16_MIN 16384
+#define LZR_K16_MIN 8192
 #endif
 uint32_t enc_warps_per_chunk(uint32_t C) {
   static int env = -1;

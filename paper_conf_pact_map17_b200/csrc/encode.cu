@@ -552,9 +552,16 @@ struct MaxThreads {
                    : (K == 2 ? 640
                              : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : (K == 16 ? 512 : LZR_K8_THREADS)))));
 };
-template <int K, bool G1 = false>
+// K = 16 outside the big layout: 2 CTAs per SM (<= 64 registers) so that two
+// 16 KiB chunks of 16 warps fit an SM; one 32 KiB chunk fills it anyway
+#ifndef LZR_K16_MINB
+#define LZR_K16_MINB 2
+#endif
+template <int K, bool G1 = false, bool BIG = false>
 struct MinBlocks {
-  static constexpr int value = G1 ? (K == 4 ? 9 : 1) : (K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : 1));
+  static constexpr int value =
+      G1 ? (K == 4 ? 9 : 1)
+         : (K == 4 ? LZR_K4_MINB : (K == 8 ? LZR_K8_MINB : (K == 16 && !BIG ? LZR_K16_MINB : 1)));
 };
 #ifndef LZR_G1_MAX_WAVES
 #define LZR_G1_MAX_WAVES 12u
@@ -562,7 +569,7 @@ struct MinBlocks {
 constexpr uint32_t kG1MaxWaves = LZR_G1_MAX_WAVES;  // launches of fewer chunk waves than this use G1
 
 template <int K, int NS, bool LZ, bool G1, bool BIG>
-__global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1>::value)
+__global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG>::value)
     lzr_encode_kernel(const EncArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
@@ -1172,7 +1179,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   if (per_sm == 0) {
     // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
-    if (MinBlocks<K, G1>::value > 1 &&
+    if (MinBlocks<K, G1, BIG>::value > 1 &&
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG>,
                                                       groups * 32 * K, smem) != cudaSuccess)
       per_sm = 1;
