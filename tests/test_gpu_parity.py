@@ -115,6 +115,8 @@ def test_adversarial_bitexact(lzr, ref, name, x):
     # in-bucket search for p's entry, walk bitmaps in global scratch
     (65536, 65536, 4, 259), (65536, 65536, 3, 258), (65536, 20000, 4, 259), (40000, 40000, 4, 259),
     (32784, 32784, 5, 100),
+    # 16-warp groups (8 KiB < C <= 32 KiB), incl. sizes that are not powers of two
+    (8208, 8000, 3, 200), (12288, 12288, 4, 259), (24576, 1000, 4, 259),
 ])
 def test_param_grid_bitexact(lzr, ref, C, W, m, M):
     p = lzr.Params(chunk_size=C, window=W, min_match=m, max_match=M)
