@@ -66,6 +66,12 @@ uint32_t enc_warps_per_chunk(uint32_t C) {
   return C > LZR_K16_MIN ? 16u : (C > 4096 ? 8u : (C >= 1024 ? 4u : 1u));
 }
 
+// big chunks: two scatter splits of 4096 buckets each (1 x B200, 1 GiB, 64 KiB
+// chunks, mix/text/zero-runs GB/s: 1 split of 8192 buckets 10.5/5.2/22.0,
+// 2 splits 11.8/5.6/32.1, 4 splits 10.5/4.9/35.7)
+#ifndef LZR_BIG_SPLITS
+#define LZR_BIG_SPLITS 2u
+#endif
 // warps that share the index scatter (each a contiguous position range with
 // its own cursor array; the hash table shrinks by the same factor)
 uint32_t enc_scatter_splits(uint32_t K, uint32_t C) {
@@ -76,7 +82,10 @@ uint32_t enc_scatter_splits(uint32_t K, uint32_t C) {
   }
   // default (config-3 sweep, 1 x B200): 1 split at K = 4 (C = 4 KiB: the full
   // C-bucket table matters more than the serial scatter), 4 at K = 8
-  if (K > 8) return C > kBigChunk ? 1u : 4u;  // big chunks: one scatter (B counters fill the slot region)
+  if (K > 8) {  // big chunks: NS splits share the slot region's 8192 counters
+    if (C > kBigChunk) return env == 2 || env == 4 ? (uint32_t)env : LZR_BIG_SPLITS;
+    return 4u;
+  }
   const uint32_t ns = env > 0 ? (uint32_t)env : (K >= 8 ? 4u : 1u);
   return K < 4 ? 1u : (ns < K ? ns : K);  // (kernels are instantiated for these)
 }

@@ -281,11 +281,15 @@ __device__ __forceinline__ uint32_t best_match(const Smem& S, uint32_t p, uint32
   if (BIG) {
     // big chunks: no slot array -- find p inside its bucket [bs, be) (entries
     // ascending) by a 32-ary search, lane i probing lo + i * step
-    const uint16_t* ends = S.slot;
+    const uint16_t* ends = S.slot + (a.L.nsplit - 1) * (1u << a.L.hbits);  // the last split's cursors
     const uint32_t h = khash(kp, a.L.hbits, a.kmask);
     const uint32_t bs = h ? ends[h - 1] : 0u;
     uint32_t lo = bs, hi = ends[h];  // p in [lo, hi), sorted[lo] <= p
+#ifdef LZR_WATCHDOG
+    uint32_t spins = 0;
+#endif
     while (hi - lo > 32u) {
+      LZR_SPIN_GUARD(spins, "bucket search")
       const uint32_t step = (hi - lo + 31u) >> 5;
       const uint32_t idx = lo + lane * step;
       const uint32_t bal = __ballot_sync(kFull, idx < hi && S.sorted[idx] <= p);
@@ -924,7 +928,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG
       const uint32_t q = S.sorted[sl];
       const uint32_t kq = ld32u(S.data, q) & a.kmask;
       const uint32_t h = khash(kq, hb, a.kmask);
-      const uint32_t bs = h ? S.slot[h - 1] : 0u;
+      const uint32_t bs = h ? S.slot[(NS - 1) * B + h - 1] : 0u;
       bool has = false;
       for (uint32_t s2 = sl; s2 > bs;) {
         const uint32_t q2 = S.sorted[--s2];
@@ -1226,8 +1230,12 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
       }
     case 16:  // chunks above 16 KiB: one group of 16 warps per SM
       if (enc_big(a.C)) {
-        if (a.L.nsplit != 1) return cudaErrorInvalidConfiguration;
-        return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+        switch (a.L.nsplit) {
+          case 1: return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+          case 2: return launch_k<16, 2, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+          case 4: return launch_k<16, 4, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+          default: return cudaErrorInvalidConfiguration;
+        }
       }
       if (a.L.nsplit != 4) return cudaErrorInvalidConfiguration;
       return launch_k<16, 4, LZ, false, false>(a, sm_count, smem_optin, s, launches);

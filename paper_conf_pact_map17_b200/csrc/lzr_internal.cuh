@@ -128,7 +128,7 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
   const bool big = enc_big(C);
   L.hbits = big ? kBigHashBits : enc_hash_bits(C);
   L.nsplit = 1;
-  while (!big && L.nsplit < NS && L.hbits > 4) {
+  while (L.nsplit < NS && L.hbits > 4) {  // (big: NS splits share the 8192 counters)
     --L.hbits;
     L.nsplit <<= 1;
   }
@@ -141,7 +141,7 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
   o += 2 * C;  // u16 positions grouped by hash bucket, ascending
   L.off_slot = o;
   // u16 histogram -> cursors -> slot of each position (big: -> bucket ends)
-  o += big ? 2 * B : 2 * (C > B ? C : B);
+  o += big ? 2 * B * L.nsplit : 2 * (C > B ? C : B);  // (NS cursor arrays of B counters)
   L.off_bm = o;
   L.bm_words = (C + 31) / 32 + 1;  // candidate / byte-change: +1 for two-word funnel reads
   L.tb_words = (C + 31) / 32;      // per-segment token-start bitmaps
