@@ -45,15 +45,19 @@ cudaError_t dev_info(DevInfo* out) {
 bool aligned(const void* p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
 // Warps cooperating on one chunk (K): 4 up to 4 KiB chunks, 8 up to 8 KiB
-// (fewer chunks fit one SM's shared memory, so each gets more warps), 16 above
-// with the walk bitmaps in the L2 scratch and <= 56 registers, so two 16 KiB
-// chunks (or one 32 KiB chunk) of 16 warps run per SM (1 x B200, 1 GiB mix,
-// GB/s: 16 KiB 25.9 -> 33.7, 32 KiB 12.0 -> 17.8; at 8 KiB 16 warps lose to
-// four groups of 8: 34.1 vs 44.0).
+// (fewer chunks fit one SM's shared memory, so each gets more warps), 16 up to
+// 16 KiB with the walk bitmaps in the L2 scratch and <= 56 registers (two
+// chunks of 16 warps per SM), 32 above (one chunk of 32 warps per SM, <= 64
+// registers).  1 x B200, 1 GiB mix, GB/s: 16 KiB 25.9 (K = 8) -> 33.7 (16) /
+// 25.6 (32); 32 KiB 12.0 (8) -> 17.8 (16) -> 24.0 (32); 64 KiB 11.8 (16) ->
+// 16.7 (32); at 8 KiB 16 warps lose to four groups of 8: 34.1 vs 44.0.
 // LZR_ENCODE_WARPS=1,2,3,4,8 overrides (tuning).
 // chunks above this size get 16 warps (walk bitmaps in the L2 scratch)
 #ifndef LZR_K16_MIN
 #define LZR_K16_MIN 8192
+#endif
+#ifndef LZR_K32_MIN
+#define LZR_K32_MIN 16384
 #endif
 uint32_t enc_warps_per_chunk(uint32_t C) {
   static int env = -1;
@@ -61,9 +65,9 @@ uint32_t enc_warps_per_chunk(uint32_t C) {
     const char* e = getenv("LZR_ENCODE_WARPS");
     env = (e && ((*e >= '1' && *e <= '4') || *e == '8')) ? (*e - '0') : 0;
   }
-  if (C > kBigChunk) return 16u;  // the big-chunk layout (lzr_internal.cuh) is built for 16
+  if (C > kBigChunk) return LZR_BIG_WARPS;  // the big-chunk layout (lzr_internal.cuh)
   if (env > 0) return (uint32_t)env;
-  return C > LZR_K16_MIN ? 16u : (C > 4096 ? 8u : (C >= 1024 ? 4u : 1u));
+  return C > LZR_K32_MIN ? 32u : (C > LZR_K16_MIN ? 16u : (C > 4096 ? 8u : (C >= 1024 ? 4u : 1u)));
 }
 
 // big chunks: two scatter splits of 4096 buckets each (1 x B200, 1 GiB, 64 KiB

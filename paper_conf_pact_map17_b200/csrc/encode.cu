@@ -554,7 +554,7 @@ struct MaxThreads {
       G1 ? 32 * K
          : (K == 1 ? 320
                    : (K == 2 ? 640
-                             : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : (K == 16 ? 512 : LZR_K8_THREADS)))));
+                             : (K == 3 ? 864 : (K == 4 ? LZR_K4_THREADS : (K == 16 ? 512 : (K == 32 ? 1024 : LZR_K8_THREADS))))));
 };
 // K = 16 outside the big layout: 2 CTAs per SM (<= 64 registers) so that two
 // 16 KiB chunks of 16 warps fit an SM; one 32 KiB chunk fills it anyway
@@ -591,8 +591,8 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG
   S.cb = bms + nw;
   S.tb = bms + 2 * nw;  // (big chunks: in the global scratch, below)
   // token-start bitmaps of the walk segments in the global scratch: big chunks
-  // and the 16-warp groups of chunks above 16 KiB
-  constexpr bool TBG = BIG || K == 16;
+  // and the 16- and 32-warp groups of chunks above 8 KiB
+  constexpr bool TBG = BIG || K >= 16;
   S.runs = TBG ? bms + 2 * nw : S.tb + K * a.L.tb_words;
   S.ctrl = S.runs + a.L.max_runs;
   S.bar = reinterpret_cast<uint64_t*>(base + a.L.off_mbar);
@@ -1228,7 +1228,14 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
         case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;
       }
-    case 16:  // chunks above 16 KiB: one group of 16 warps per SM
+    case 32:  // chunks above 16 KiB: one group of 32 warps per SM
+      if (enc_big(a.C)) {
+        if (a.L.nsplit != 2) return cudaErrorInvalidConfiguration;
+        return launch_k<32, 2, LZ, false, true>(a, sm_count, smem_optin, s, launches);
+      }
+      if (a.L.nsplit != 4) return cudaErrorInvalidConfiguration;
+      return launch_k<32, 4, LZ, false, false>(a, sm_count, smem_optin, s, launches);
+    case 16:  // 8 KiB < C <= 16 KiB: groups of 16 warps, two per SM
       if (enc_big(a.C)) {
         switch (a.L.nsplit) {
           case 1: return launch_k<16, 1, LZ, false, true>(a, sm_count, smem_optin, s, launches);

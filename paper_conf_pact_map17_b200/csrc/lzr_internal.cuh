@@ -109,6 +109,9 @@ struct EncLayout {
 #define LZR_BIG_CHUNK 32768
 #endif
 constexpr uint32_t kBigChunk = LZR_BIG_CHUNK;
+#ifndef LZR_BIG_WARPS
+#define LZR_BIG_WARPS 32u
+#endif
 constexpr uint32_t kBigHashBits = 13;
 
 __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
@@ -148,7 +151,7 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
   // candidate, byte-change, K token-start bitmaps (big: in global scratch); run
   // list; ctrl (4 + 2K words)
   L.max_runs = enc_max_runs(C);
-  const bool tbg = big || K == 16;  // walk bitmaps in the global scratch
+  const bool tbg = big || K >= 16;  // walk bitmaps in the global scratch
   o += 4 * (2 * L.bm_words + (tbg ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K);
   o = align_up(o, 8);
   L.off_mbar = o;
@@ -160,7 +163,7 @@ __host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t
 // global scratch bytes per resident group: (d-1) per position (u16), + the K
 // token-start bitmaps when big
 __host__ __device__ inline size_t enc_scratch_per_group(const EncLayout& L, uint32_t C) {
-  return (enc_big(C) || L.K == 16) ? align_up_z(2 * (size_t)C + 4 * (size_t)L.K * L.tb_words, 256)
+  return (enc_big(C) || L.K >= 16) ? align_up_z(2 * (size_t)C + 4 * (size_t)L.K * L.tb_words, 256)
                                    : 2 * (size_t)C;
 }
 
