@@ -257,6 +257,22 @@ def test_compress_host_pipeline(lzr, ref, n):
         assert np.array_equal(h_out[:tot].numpy(), g_out)
 
 
+@pytest.mark.parametrize("C", [16384, 32768, 65536])
+def test_compress_host_pipeline_large_chunks(lzr, ref, C):
+    """The host pipeline with 16- and 32-warp groups (walk bitmaps in the L2
+    scratch of every batch's workspace) == the device path == the oracle."""
+    n = C * 13 + 4112
+    x = synth.fill_host(n, C, "mix", seed=C)
+    p = lzr.Params(chunk_size=C)
+    h = torch.from_numpy(x).pin_memory()
+    h_out, h_sizes, h_offs, tot = lzr.compress_host(h, p, batch_bytes=4 * C)
+    r_out, r_sizes, r_offs, r_tot = ref.compress(x, _ref_params(ref, p))
+    assert tot == r_tot
+    assert np.array_equal(h_sizes.numpy().view(np.uint32), r_sizes)
+    assert np.array_equal(h_offs.numpy().view(np.uint64), r_offs)
+    assert np.array_equal(h_out[:tot].numpy(), r_out)
+
+
 def test_empty_input(lzr):
     xd = torch.empty(0, dtype=torch.uint8, device="cuda")
     out, sizes, offs, total = lzr.compress(xd, lzr.Params())
