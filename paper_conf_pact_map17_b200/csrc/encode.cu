@@ -398,13 +398,15 @@ __device__ __forceinline__ void walk_segment(const Smem& S, uint16_t* d1, uint32
       uint32_t l = r >> 16;
       // LZ: a longer match at q + 1 is possible only if l is below its cap
       // min(M, n - q - 1) and q + 1 has a same-key candidate
-      // A match longer than l at q + 1 also covers the key at s = q + l + 2 - k
-      // (the last key inside it that a match of length l + 1 must contain), at
-      // the same distance: s then has a candidate.  No candidate at s (and s a
-      // candidate-tracked position, s < P) => no longer match => no search.
-      const uint32_t s_lz = q + l + 2 - a.kbytes;
+      // A match longer than l at q + 1 covers the keys at s = q + l + 1 - k and
+      // q + l + 2 - k (the keys that contain x[q + l], the byte that ended q's
+      // match; k = key length), at its own distance: both then have a
+      // candidate.  Either without one (and a candidate-tracked position,
+      // < P) => no longer match at q + 1 => no search.
+      const uint32_t s_lz = q + l + 1 - a.kbytes;
+      const uint32_t two = __funnelshift_r(S.cand[s_lz >> 5], S.cand[(s_lz >> 5) + 1], s_lz & 31u) & 3u;
       if (LZ && l >= a.m && l < min(a.M, n - q - 1) && ((S.cand[(q + 1) >> 5] >> ((q + 1) & 31u)) & 1u) &&
-          (s_lz >= P || ((S.cand[s_lz >> 5] >> (s_lz & 31u)) & 1u))) {
+          (s_lz + 1 >= P || two == 3u)) {
         cr = best_match<BIG>(S, q + 1, n, nruns, a, lane, l, S.data[q]);  // exact if > l
         cq = q + 1;
         if ((cr >> 16) > l) l = 0;  // deferred: x[q] is a literal
