@@ -821,6 +821,25 @@ def main():
             e2e_t.append(time.perf_counter() - t0)
         e2e_s = R.reduce(statistics.median(e2e_t), "max")
         e2e_v = n_e2e * world / e2e_s / 1e9
+        # the read path end to end: lzr_decompress_host of what was just written
+        d_t, dec_ok = [], True
+        scratch_d = torch.empty(max(256, lzr.lib().lzr_decompress_host_scratch_bytes(
+            16 << 20, ctypes.byref(p.c()))), dtype=torch.uint8, device=dev)
+        h_y = torch.empty(n_e2e, dtype=torch.uint8, pin_memory=True)
+        lzr.decompress_host(h_out, h_sizes, h_offs, n_e2e, p, 16 << 20, scratch_d, h_y)  # warm-up
+        for _ in range(max(1, min(a.steps, 5))):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            _, derr_h = lzr.decompress_host(h_out, h_sizes, h_offs, n_e2e, p, 16 << 20, scratch_d, h_y)
+            d_t.append(time.perf_counter() - t0)
+            dec_ok = dec_ok and derr_h == 0
+        dec_ok = dec_ok and bool(torch.equal(h_y, hx))
+        d_s = R.reduce(statistics.median(d_t), "max")
+        line["decode_e2e"] = {"value": round(n_e2e * world / d_s / 1e9, 4), "unit": "GB/s (output)",
+                              "h2d_bytes_per_step": int(tot) + 12 * n_e2e_chunks, "d2h_bytes_per_step": n_e2e,
+                              "round_trip": "ok" if dec_ok else "MISMATCH",
+                              "api": "lzr_decompress_host (pinned host in/out, 16 MiB batches, 3 buffer sets, shared H2D / D2H copy streams)"}
+        del scratch_d
         line["e2e"] = {"value": round(e2e_v, 4), "unit": UNIT, "h2d_bytes_per_step": n_e2e,
                        "d2h_bytes_per_step": int(tot) + 12 * n_e2e_chunks,
                        "api": "lzr_compress_host (pinned host in/out, 16 MiB batches, 3 buffer sets, shared H2D / D2H copy streams)"

@@ -18,7 +18,7 @@ from dataclasses import dataclass
 __all__ = [
     "Params", "LzrError", "lib", "num_chunks", "compress_bound", "compress_workspace_bytes",
     "compress", "compress_encode", "compress_compact", "scan_sizes", "decompress",
-    "compress_host", "validate_params", "status_str", "last_launch_count",
+    "compress_host", "decompress_host", "validate_params", "status_str", "last_launch_count",
     "fingerprint", "DedupIndex", "gather_chunks", "dedup_compress", "owner_counts", "route",
     "unroute",
 ]
@@ -37,7 +37,7 @@ EXPORTED_SYMBOLS = [
     "lzr_compress_host_scratch_bytes", "lzr_compress_host", "lzr_status_str",
     "lzr_last_launch_count", "lzr_fingerprint_chunks", "lzr_dedup_table_bytes", "lzr_dedup_index",
     "lzr_gather_chunks", "lzr_dedup_index_gidx", "lzr_dedup_owner_counts", "lzr_dedup_route",
-    "lzr_dedup_unroute",
+    "lzr_dedup_unroute", "lzr_decompress_host_scratch_bytes", "lzr_decompress_host",
 ]
 
 
@@ -100,6 +100,9 @@ def lib():
         L.lzr_compress_host_scratch_bytes.argtypes = [sz, P]
         L.lzr_compress_host_scratch_bytes.restype = sz
         L.lzr_compress_host.argtypes = [vp, sz, P, vp, sz, vp, vp, vp, sz, vp, sz]
+        L.lzr_decompress_host_scratch_bytes.argtypes = [sz, P]
+        L.lzr_decompress_host_scratch_bytes.restype = sz
+        L.lzr_decompress_host.argtypes = [vp, vp, vp, sz, P, vp, vp, sz, vp, sz]
         L.lzr_status_str.argtypes = [ctypes.c_int]
         L.lzr_status_str.restype = ctypes.c_char_p
         L.lzr_last_launch_count.argtypes = []
@@ -318,6 +321,31 @@ def compress_host(h_in, p: Params = Params(), batch_bytes: int = 16 << 20, scrat
         ctypes.byref(tot), batch_bytes, _ptr(scratch), scratch.numel())
     _check(st, "lzr_compress_host")
     return h_out, h_sizes[:N], h_offsets[:N], tot.value
+
+
+def decompress_host(h_comp, h_sizes, h_offsets, n: int, p: Params = Params(), batch_bytes: int = 16 << 20,
+                    scratch=None, h_out=None):
+    """End-to-end decompression of host (preferably pinned) buffers through the
+    C ABI's host pipeline (H2D of each batch's streams, decode, D2H inside).
+    Synchronous.  Returns (h_out, error): error 0 or 1 + index of the first
+    corrupt chunk."""
+    import torch
+
+    batch_bytes = -(-batch_bytes // p.chunk_size) * p.chunk_size
+    if batch_bytes == 0 or batch_bytes > n:
+        batch_bytes = max(p.chunk_size, -(-n // p.chunk_size) * p.chunk_size)
+    need = lib().lzr_decompress_host_scratch_bytes(batch_bytes, ctypes.byref(p.c()))
+    if scratch is None or scratch.numel() < need:
+        scratch = torch.empty(max(256, need), dtype=torch.uint8, device="cuda")
+    if h_out is None:
+        h_out = torch.empty(max(1, n), dtype=torch.uint8, pin_memory=True)
+    err = ctypes.c_int32()
+    st = lib().lzr_decompress_host(
+        ctypes.c_void_p(h_comp.data_ptr()), ctypes.c_void_p(h_sizes.data_ptr()),
+        ctypes.c_void_p(h_offsets.data_ptr()), n, ctypes.byref(p.c()), ctypes.c_void_p(h_out.data_ptr()),
+        ctypes.byref(err), batch_bytes, _ptr(scratch), scratch.numel())
+    _check(st, "lzr_decompress_host")
+    return h_out[:n], err.value
 
 
 # ---- dedup upstream of compression (include/lzr.h; DESIGN.md §11) ---------------

@@ -672,3 +672,134 @@ int lzr_compress_host(const void* h_in, size_t n_bytes, const lzr_params* p, voi
 }
 
 }  // extern "C"
+
+// ---- host-buffer decompression (the read path's end-to-end call) -----------
+
+namespace {
+struct DecSet {
+  uint8_t *comp, *out;
+  uint32_t* sizes;
+  uint64_t* offs;
+  int32_t* err;
+};
+
+size_t dec_set_bytes(size_t batch, const lzr_params* p) {
+  const size_t C = p->chunk_size;
+  const size_t N = (batch + C - 1) / C;
+  return 2 * align_up_z(batch, 256) + align_up_z(4 * N, 256) + align_up_z(8 * N, 256) + 256;
+}
+
+DecSet dec_carve(uint8_t* base, size_t batch, const lzr_params* p) {
+  const size_t C = p->chunk_size;
+  const size_t N = (batch + C - 1) / C;
+  DecSet d;
+  size_t o = 0;
+  d.comp = base + o; o += align_up_z(batch, 256);
+  d.out = base + o; o += align_up_z(batch, 256);
+  d.sizes = (uint32_t*)(base + o); o += align_up_z(4 * N, 256);
+  d.offs = (uint64_t*)(base + o); o += align_up_z(8 * N, 256);
+  d.err = (int32_t*)(base + o);
+  return d;
+}
+}  // namespace
+
+extern "C" {
+
+size_t lzr_decompress_host_scratch_bytes(size_t batch_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK || batch_bytes == 0) return 0;
+  return host_sets() * align_up_z(dec_set_bytes(batch_bytes, p), 256);
+}
+
+int lzr_decompress_host(const void* h_comp, const uint32_t* h_sizes, const uint64_t* h_offsets,
+                        size_t n_bytes, const lzr_params* p, void* h_out, int32_t* h_error,
+                        size_t batch_bytes, void* d_scratch, size_t scratch_bytes) {
+  int st = lzr_validate_params(p);
+  if (st) return st;
+  const size_t C = p->chunk_size;
+  if (h_error) *h_error = 0;
+  if (n_bytes == 0) return LZR_OK;
+  if (!h_comp || !h_sizes || !h_offsets || !h_out || !d_scratch) return LZR_ERR_INVALID_ARG;
+  if (batch_bytes == 0) batch_bytes = align_up_z(n_bytes, C);
+  if (batch_bytes % C) return LZR_ERR_INVALID_ARG;
+  if (!aligned(d_scratch, 256)) return LZR_ERR_INVALID_ARG;
+  DevInfo di;
+  if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
+  const size_t per = align_up_z(dec_set_bytes(batch_bytes, p), 256);
+  const int nsets = host_sets();
+  if (scratch_bytes < nsets * per) return LZR_ERR_CAPACITY;
+  const size_t nb = (n_bytes + batch_bytes - 1) / batch_bytes;
+  const size_t cpb = batch_bytes / C;
+  HostStreams* hs = acquire_host_streams(nsets);
+  if (!hs) return LZR_ERR_CUDA;
+  // one H2D stream, one D2H stream (copies in batch order at full link rate),
+  // a compute stream per buffer set; events order the reuse of a set's
+  // buffers.  One error word for the whole call (set 0's), every batch's
+  // kernel reporting global chunk indices (err_base), initialised before the
+  // first decode and fixed up after the last.
+  cudaStream_t h2d = hs->cin[0], d2h = nsets > 1 ? hs->cin[1] : hs->cin[0];
+  int32_t* derr = dec_carve((uint8_t*)d_scratch, batch_bytes, p).err;
+  int rc = LZR_OK;
+  int launches = 0;
+  if (decode_err_init(derr, hs->s[0]) != cudaSuccess || cudaEventRecord(hs->ev_in[0], hs->s[0]) != cudaSuccess)
+    rc = LZR_ERR_CUDA;
+  for (int k = 1; k < nsets && rc == LZR_OK; ++k)
+    if (cudaStreamWaitEvent(hs->s[k], hs->ev_in[0], 0) != cudaSuccess) rc = LZR_ERR_CUDA;
+  for (size_t b = 0; b < nb && rc == LZR_OK; ++b) {
+    const int k = (int)(b % nsets);
+    DecSet d = dec_carve((uint8_t*)d_scratch + k * per, batch_bytes, p);
+    const size_t c0 = b * cpb;
+    const size_t len = n_bytes - b * batch_bytes < batch_bytes ? n_bytes - b * batch_bytes : batch_bytes;
+    const size_t N = (len + C - 1) / C;
+    // the batch's compressed bytes: the span [lo, hi) of its chunks' streams
+    // (any offsets are allowed; compacted streams always fit the buffer)
+    uint64_t lo = ~0ull, hi = 0;
+    for (size_t i = 0; i < N; ++i) {
+      const uint64_t o = h_offsets[c0 + i], e = o + h_sizes[c0 + i];
+      if (o < lo) lo = o;
+      if (e > hi) hi = e;
+    }
+    if (hi - lo > batch_bytes) {
+      rc = LZR_ERR_CAPACITY;
+      break;
+    }
+    cudaStream_t ss = hs->s[k];
+    // H2D once the set's previous decode has read its inputs
+    if ((b >= (size_t)nsets && cudaStreamWaitEvent(h2d, hs->ev_kdone[k], 0) != cudaSuccess) ||
+        (hi > lo && cudaMemcpyAsync(d.comp, (const uint8_t*)h_comp + lo, hi - lo, cudaMemcpyHostToDevice, h2d) != cudaSuccess) ||
+        cudaMemcpyAsync(d.sizes, h_sizes + c0, 4 * N, cudaMemcpyHostToDevice, h2d) != cudaSuccess ||
+        cudaMemcpyAsync(d.offs, h_offsets + c0, 8 * N, cudaMemcpyHostToDevice, h2d) != cudaSuccess ||
+        cudaEventRecord(hs->ev_in[k], h2d) != cudaSuccess || cudaStreamWaitEvent(ss, hs->ev_in[k], 0) != cudaSuccess ||
+        // the decode rewrites the set's output buffer once its previous D2H is done
+        (b >= (size_t)nsets && cudaStreamWaitEvent(ss, hs->ev_out[k], 0) != cudaSuccess)) {
+      rc = LZR_ERR_CUDA;
+      break;
+    }
+    // offsets are the stream's own: the batch buffer stands at offset lo
+    int l = 0;
+    if (launch_decode(d.comp - lo, d.sizes, d.offs, len, (uint32_t)C, p->min_match, d.out, derr,
+                      di.sm_count, di.smem_optin, ss, &l, c0, false) != cudaSuccess ||
+        cudaEventRecord(hs->ev_kdone[k], ss) != cudaSuccess || cudaStreamWaitEvent(d2h, hs->ev_kdone[k], 0) != cudaSuccess ||
+        cudaMemcpyAsync((uint8_t*)h_out + b * batch_bytes, d.out, len, cudaMemcpyDeviceToHost, d2h) != cudaSuccess ||
+        cudaEventRecord(hs->ev_out[k], d2h) != cudaSuccess) {
+      rc = LZR_ERR_CUDA;
+      break;
+    }
+    launches += l;
+  }
+  // every decode done -> fix the error word up and read it back
+  for (int k = 0; k < nsets; ++k)
+    if (cudaStreamSynchronize(hs->s[k]) != cudaSuccess && rc == LZR_OK) rc = LZR_ERR_CUDA;
+  int32_t e_host = 0;
+  if (rc == LZR_OK && (decode_err_fini(derr, hs->s[0], &launches) != cudaSuccess ||
+                       cudaMemcpyAsync(&e_host, derr, 4, cudaMemcpyDeviceToHost, hs->s[0]) != cudaSuccess))
+    rc = LZR_ERR_CUDA;
+  if ((cudaStreamSynchronize(hs->s[0]) != cudaSuccess || cudaStreamSynchronize(h2d) != cudaSuccess ||
+       cudaStreamSynchronize(d2h) != cudaSuccess) && rc == LZR_OK)
+    rc = LZR_ERR_CUDA;
+  release_host_streams(hs);
+  if (h_error) *h_error = rc == LZR_OK ? e_host : 0;
+  t_launches = launches;
+  return rc;
+}
+
+}  // extern "C"

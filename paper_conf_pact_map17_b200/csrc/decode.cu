@@ -64,7 +64,7 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
 __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_kernel(
     const uint8_t* __restrict__ comp, const uint32_t* __restrict__ sizes,
     const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C, uint32_t m,
-    uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride) {
+    uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride, uint64_t err_base) {
   extern __shared__ __align__(16) uint8_t dsm[];
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   uint8_t* obuf = dsm + (size_t)warp * buf_stride;  // rebuilt chunk (C bytes)
@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
     }
     if (!bad && ip != S) bad = true;
     if (bad) {
-      if (lane == 0 && err) atomicMin(err, (int32_t)(c + 1));
+      if (lane == 0 && err) atomicMin(err, (int32_t)(c + 1 + err_base));
       __syncwarp();
       continue;
     }
@@ -226,12 +226,23 @@ __global__ void lzr_decode_fixup_kernel(int32_t* err) {
 
 }  // namespace
 
+cudaError_t decode_err_init(int32_t* err, cudaStream_t s) {
+  return cudaMemsetAsync(err, 0x7F, sizeof(int32_t), s);
+}
+
+cudaError_t decode_err_fini(int32_t* err, cudaStream_t s, int* launches) {
+  lzr_decode_fixup_kernel<<<1, 1, 0, s>>>(err);
+  if (launches) ++*launches;
+  return cudaGetLastError();
+}
+
 cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,
                           size_t n_bytes, uint32_t C, uint32_t m, uint8_t* out, int32_t* err,
-                          int sm_count, int smem_optin, cudaStream_t s, int* launches) {
+                          int sm_count, int smem_optin, cudaStream_t s, int* launches,
+                          uint64_t err_base, bool err_own) {
   const size_t N = (n_bytes + C - 1) / C;
   if (N == 0) {
-    if (err) return cudaMemsetAsync(err, 0, sizeof(int32_t), s);
+    if (err && err_own) return cudaMemsetAsync(err, 0, sizeof(int32_t), s);
     return cudaSuccess;
   }
   const uint32_t stride = align_up(C, 16);  // rebuilt chunk
@@ -282,23 +293,19 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
     cache[dev].per_sm = per_sm;
   }
   int32_t* errp = err;
-  if (errp) {
-    e = cudaMemsetAsync(errp, 0x7F, sizeof(int32_t), s);
+  if (errp && err_own) {
+    e = decode_err_init(errp, s);
     if (e != cudaSuccess) return e;
   }
   size_t blocks = (N + warps - 1) / warps;
   const size_t cap = (size_t)sm_count * per_sm;
   if (LZR_DEC_ONEWAVE && blocks > cap) blocks = cap;
   lzr_decode_kernel<<<(unsigned)blocks, warps * 32, smem, s>>>(comp, sizes, offsets, n_bytes, C, m,
-                                                              out, errp, N, stride);
+                                                              out, errp, N, stride, err_base);
   if (launches) ++*launches;
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  if (err) {
-    lzr_decode_fixup_kernel<<<1, 1, 0, s>>>(err);
-    if (launches) ++*launches;
-    e = cudaGetLastError();
-  }
+  if (err && err_own) e = decode_err_fini(err, s, launches);
   return e;
 }
 

@@ -199,9 +199,16 @@ cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const 
                            size_t slot_stride,
                            const uint32_t* sizes, const uint64_t* offsets, uint8_t* out,
                            int sm_count, cudaStream_t s, int* launches);
+// decode: err (optional) receives min(1 + err_base + chunk) over corrupt
+// chunks; err_own: this launch initialises it (0x7F7F7F7F) and fixes it up to
+// 0 when nothing was corrupt -- otherwise the caller does both
+// (decode_err_init / decode_err_fini) around several launches sharing it
 cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,
                           size_t n_bytes, uint32_t C, uint32_t m, uint8_t* out, int32_t* err,
-                          int sm_count, int smem_optin, cudaStream_t s, int* launches);
+                          int sm_count, int smem_optin, cudaStream_t s, int* launches,
+                          uint64_t err_base = 0, bool err_own = true);
+cudaError_t decode_err_init(int32_t* err, cudaStream_t s);
+cudaError_t decode_err_fini(int32_t* err, cudaStream_t s, int* launches);
 
 // dedup.cu
 cudaError_t launch_sha1(const uint8_t* in, size_t n, uint32_t C, uint8_t* fp, cudaStream_t s,

@@ -95,6 +95,16 @@ def test_host_argument_errors(lzr):
     assert L.lzr_validate_params(ctypes.byref(lzr.Params(parse=2).c())) == lzr.ERR_UNSUPPORTED
     # n == 0 is a no-op
     assert L.lzr_compress_encode(None, 0, cp, None, None, 0, None) == lzr.OK
+    # host-buffer decompression: n == 0 no-op (error word cleared), NULL
+    # buffers / a batch that is not a multiple of C rejected before any CUDA call
+    err = ctypes.c_int32(7)
+    assert L.lzr_decompress_host(None, None, None, 0, cp, None, ctypes.byref(err), 0, None, 0) == lzr.OK
+    assert err.value == 0
+    v = ctypes.c_void_p(256)
+    assert L.lzr_decompress_host(None, v, v, 4096, cp, v, None, 0, v, 1 << 30) == lzr.ERR_INVALID_ARG
+    assert L.lzr_decompress_host(v, v, v, 8192, cp, v, None, 4000, v, 1 << 30) == lzr.ERR_INVALID_ARG
+    assert L.lzr_decompress_host_scratch_bytes(1 << 20, cp) > 2 * (1 << 20)
+    assert L.lzr_decompress_host_scratch_bytes(0, cp) == 0
 
 
 def test_no_gpu_fails_loudly(lzr):

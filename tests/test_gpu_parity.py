@@ -273,6 +273,32 @@ def test_compress_host_pipeline_large_chunks(lzr, ref, C):
     assert np.array_equal(h_out[:tot].numpy(), r_out)
 
 
+@pytest.mark.parametrize("C,batch", [(4096, 0), (4096, 1 << 20), (4096, 3 * 4096 * 7), (16384, 4 * 16384),
+                                     (65536, 2 * 65536)])
+def test_decompress_host_pipeline(lzr, ref, C, batch):
+    """lzr_decompress_host (H2D of each batch's streams, decode, D2H) inverts
+    lzr_compress_host, ragged tail included; a corrupted stream is reported at
+    the same chunk as the oracle's decoder reports it."""
+    n = C * 37 + 1000
+    x = synth.fill_host(n, C, "mix", seed=C + batch)
+    p = lzr.Params(chunk_size=C)
+    h = torch.from_numpy(x).pin_memory()
+    h_out, h_sizes, h_offs, tot = lzr.compress_host(h, p, batch_bytes=1 << 20)
+    y, err = lzr.decompress_host(h_out, h_sizes, h_offs, n, p, batch_bytes=batch)
+    assert err == 0 and np.array_equal(y.numpy(), x)
+    # corrupt one compressed (non-raw) chunk in a later batch: same verdict as the oracle
+    sz = h_sizes.numpy().view(np.uint32)
+    nonraw = [i for i in range(sz.size) if sz[i] < min(C, n - i * C)]
+    i = nonraw[len(nonraw) // 2]
+    bad = h_out.clone()
+    o = int(h_offs.numpy().view(np.uint64)[i])
+    bad[o] ^= 0xFF  # the first flag byte: token kinds change
+    r_st, r_bad, _ = ref.decompress(bad.numpy()[: int(tot)], sz, h_offs.numpy().view(np.uint64), n,
+                                    ref.Params(chunk_size=C))
+    _, err2 = lzr.decompress_host(bad, h_sizes, h_offs, n, p, batch_bytes=batch)
+    assert err2 == r_bad
+
+
 def test_empty_input(lzr):
     xd = torch.empty(0, dtype=torch.uint8, device="cuda")
     out, sizes, offs, total = lzr.compress(xd, lzr.Params())
