@@ -495,3 +495,19 @@ def test_big_chunk_edge_inputs(lzr, ref):
     words = [bytes(rng.integers(97, 123, int(rng.integers(3, 9)), dtype=np.uint8)) for _ in range(40)]
     t = b" ".join(words[int(i)] for i in rng.integers(0, 40, 30000))[: C * 2 - 5]
     _check_full(lzr, ref, np.frombuffer(t, np.uint8).copy(), lzr.Params(chunk_size=C))
+
+
+@pytest.mark.parametrize("seed", range(32))
+def test_random_params_fuzz(lzr, ref, seed):
+    """Seeded random (C, W, m, M, parse, class) configurations across every
+    kernel family (1..32 warps per chunk, the big layout) vs the oracle."""
+    rng = np.random.default_rng(1000 + seed)
+    C = int(rng.choice([16, 48, 512, 1024, 2064, 4096, 6144, 8192, 12288, 16384, 20480, 32768, 49152, 65536]))
+    W = int(rng.integers(1, C + 1)) if rng.random() < 0.5 else C
+    m = int(rng.integers(3, 8))
+    M = m + int(rng.integers(0, 256))
+    parse = int(rng.integers(0, 2))
+    cls = str(rng.choice(["mix", "text", "zeroruns", "cr2"]))
+    n = int(C * rng.integers(2, 5) + rng.integers(0, C))
+    x = synth.fill_host(n, C, cls, seed=seed)
+    _check_full(lzr, ref, x, lzr.Params(chunk_size=C, window=W, min_match=m, max_match=M, parse=parse))
