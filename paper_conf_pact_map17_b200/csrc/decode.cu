@@ -40,7 +40,12 @@ namespace {
 #define LZR_DEC_MINB 24
 #endif
 constexpr int32_t kNoError = 0x7F7F7F7F;
-constexpr uint32_t kLaneCopyMax = 16;  // matches up to this length: one lane, byte-serial
+// (1 x B200, 256 MiB, mix/text GB/s: 8 -> 347/208, 12 -> 392/241, 16 ->
+// 402/248, 24 -> 404/250; byte-serial copies 4 at a time with d >= 4: 389/234)
+#ifndef LZR_DEC_LANE_MAX
+#define LZR_DEC_LANE_MAX 16
+#endif
+constexpr uint32_t kLaneCopyMax = LZR_DEC_LANE_MAX;  // matches up to this length: one lane, byte-serial
 // (measured and not kept, 1 x B200, 256 MiB, output GB/s mix/text/zero-runs:
 // an L1 prefetch of the stream's lines at chunk start 356/247/702 vs
 // 386/247/667; short matches copied 4 source bytes per step from two aligned
