@@ -580,9 +580,18 @@ struct MinBlocks {
 #endif
 constexpr uint32_t kG1MaxWaves = LZR_G1_MAX_WAVES;  // launches of fewer chunk waves than this use G1
 
-template <int K, int NS, bool LZ, bool G1, bool BIG>
+// CF != 0: the kernel specialised for chunk size CF (the layout's offsets and
+// sizes become compile-time constants)
+template <int K, int NS, bool LZ, bool G1, bool BIG, uint32_t CF>
 __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG>::value)
-    lzr_encode_kernel(const EncArgs a) {
+    lzr_encode_kernel(const EncArgs a_in) {
+  EncArgs a_fix = a_in;
+  if (CF) {
+    constexpr EncLayout LF = enc_layout(CF ? CF : 4096u, K, NS);
+    a_fix.L = LF;
+    a_fix.C = CF;
+  }
+  const EncArgs& a = CF ? a_fix : a_in;
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t lane = threadIdx.x & 31u;
   const uint32_t warp = threadIdx.x >> 5;
@@ -1153,7 +1162,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG
   }
 }
 
-template <int K, int NS, bool LZ, bool G1 = false, bool BIG = false>
+template <int K, int NS, bool LZ, bool G1 = false, bool BIG = false, uint32_t CF = 0>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
   const int max_groups = MaxThreads<K, G1>::value / (32 * K);
@@ -1181,7 +1190,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   {
     std::lock_guard<std::mutex> lk(mu);
     if (!cache[dev].attr) {
-      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1, BIG>,
+      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1, BIG, CF>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
       if (err != cudaSuccess) return err;
       cache[dev].attr = true;
@@ -1192,7 +1201,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
     // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
     if (MinBlocks<K, G1, BIG>::value > 1 &&
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG>,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG, CF>,
                                                       groups * 32 * K, smem) != cudaSuccess)
       per_sm = 1;
     if (per_sm < 1) per_sm = 1;
@@ -1203,7 +1212,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
-  lzr_encode_kernel<K, NS, LZ, G1, BIG><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS, LZ, G1, BIG, CF><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -1230,8 +1239,10 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
         case 1:
           // few waves of chunks: one group per CTA (see MaxThreads)
           if (a.N < kG1MaxWaves * 9u * (uint32_t)sm_count)
-            return launch_k<4, 1, LZ, true>(a, sm_count, smem_optin, s, launches);
-          return launch_k<4, 1, LZ>(a, sm_count, smem_optin, s, launches);
+            return a.C == 4096 ? launch_k<4, 1, LZ, true, false, 4096>(a, sm_count, smem_optin, s, launches)
+                               : launch_k<4, 1, LZ, true>(a, sm_count, smem_optin, s, launches);
+          return a.C == 4096 ? launch_k<4, 1, LZ, false, false, 4096>(a, sm_count, smem_optin, s, launches)
+                             : launch_k<4, 1, LZ>(a, sm_count, smem_optin, s, launches);
         case 2: return launch_k<4, 2, LZ>(a, sm_count, smem_optin, s, launches);
         case 4: return launch_k<4, 4, LZ>(a, sm_count, smem_optin, s, launches);
         default: return cudaErrorInvalidConfiguration;

@@ -87,7 +87,7 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
 // ---- encode kernel shared-memory layout (one region per group of K warps) ---
 // run list capacity per chunk (runs of one byte value of length >= k): about
 // one zero run per 128 bytes of chunk (the zero-runs class has one per ~300 B)
-__host__ __device__ inline uint32_t enc_max_runs(uint32_t C) {
+__host__ __device__ constexpr uint32_t enc_max_runs(uint32_t C) {
   const uint32_t r = (C / 128 + 7) & ~7u;
   return r < 24 ? 24 : r;
 }
@@ -114,7 +114,7 @@ constexpr uint32_t kBigChunk = LZR_BIG_CHUNK;
 #endif
 constexpr uint32_t kBigHashBits = 13;
 
-__host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
+__host__ __device__ constexpr uint32_t enc_hash_bits(uint32_t C) {
   uint32_t hb = 0;
   while ((2u << hb) <= C && hb < 15) ++hb;  // largest power of two <= C (the table lives in 2C bytes)
   return hb;
@@ -123,10 +123,10 @@ __host__ __device__ inline uint32_t enc_hash_bits(uint32_t C) {
 // K warps per chunk; NS of them share the index scatter, each with its own
 // cursor array, so NS * B u16 counters must fit the 2 max(C, B)-byte slot
 // region: B = (largest power of two <= C) / NS
-__host__ __device__ inline bool enc_big(uint32_t C) { return C > kBigChunk; }
+__host__ __device__ constexpr bool enc_big(uint32_t C) { return C > kBigChunk; }
 
-__host__ __device__ inline EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t NS) {
-  EncLayout L;
+__host__ __device__ constexpr EncLayout enc_layout(uint32_t C, uint32_t K, uint32_t NS) {
+  EncLayout L{};
   L.K = K;
   const bool big = enc_big(C);
   L.hbits = big ? kBigHashBits : enc_hash_bits(C);
