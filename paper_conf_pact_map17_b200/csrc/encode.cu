@@ -581,8 +581,9 @@ struct MinBlocks {
 constexpr uint32_t kG1MaxWaves = LZR_G1_MAX_WAVES;  // launches of fewer chunk waves than this use G1
 
 // CF != 0: the kernel specialised for chunk size CF (the layout's offsets and
-// sizes become compile-time constants)
-template <int K, int NS, bool LZ, bool G1, bool BIG, uint32_t CF>
+// sizes become compile-time constants); DEF: also for the configs' parameters
+// W = C, m = 4, M = 259
+template <int K, int NS, bool LZ, bool G1, bool BIG, uint32_t CF, bool DEF = false>
 __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG>::value)
     lzr_encode_kernel(const EncArgs a_in) {
   EncArgs a_fix = a_in;
@@ -590,6 +591,13 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG
     constexpr EncLayout LF = enc_layout(CF ? CF : 4096u, K, NS);
     a_fix.L = LF;
     a_fix.C = CF;
+    if (DEF) {
+      a_fix.W = CF;
+      a_fix.m = 4;
+      a_fix.M = 259;
+      a_fix.kbytes = 4;
+      a_fix.kmask = 0xFFFFFFFFu;
+    }
   }
   const EncArgs& a = CF ? a_fix : a_in;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -1162,7 +1170,7 @@ __global__ void __launch_bounds__(MaxThreads<K, G1>::value, MinBlocks<K, G1, BIG
   }
 }
 
-template <int K, int NS, bool LZ, bool G1 = false, bool BIG = false, uint32_t CF = 0>
+template <int K, int NS, bool LZ, bool G1 = false, bool BIG = false, uint32_t CF = 0, bool DEF = false>
 cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_t s, int* launches) {
   int groups = smem_optin / (int)a.L.per_group;
   const int max_groups = MaxThreads<K, G1>::value / (32 * K);
@@ -1190,7 +1198,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   {
     std::lock_guard<std::mutex> lk(mu);
     if (!cache[dev].attr) {
-      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1, BIG, CF>,
+      err = cudaFuncSetAttribute(lzr_encode_kernel<K, NS, LZ, G1, BIG, CF, DEF>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
       if (err != cudaSuccess) return err;
       cache[dev].attr = true;
@@ -1201,7 +1209,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
     // persistent grid: every resident CTA (one per SM unless MinBlocks > 1)
     per_sm = 1;
     if (MinBlocks<K, G1, BIG>::value > 1 &&
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG, CF>,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_encode_kernel<K, NS, LZ, G1, BIG, CF, DEF>,
                                                       groups * 32 * K, smem) != cudaSuccess)
       per_sm = 1;
     if (per_sm < 1) per_sm = 1;
@@ -1212,7 +1220,7 @@ cudaError_t launch_k(const EncArgs& a, int sm_count, int smem_optin, cudaStream_
   const uint32_t need = (a.N + groups - 1) / groups;
   const uint32_t cap = (uint32_t)(sm_count * per_sm);
   const uint32_t grid = need < cap ? need : cap;
-  lzr_encode_kernel<K, NS, LZ, G1, BIG, CF><<<grid, groups * 32 * K, smem, s>>>(a);
+  lzr_encode_kernel<K, NS, LZ, G1, BIG, CF, DEF><<<grid, groups * 32 * K, smem, s>>>(a);
   if (launches) ++*launches;
   return cudaGetLastError();
 }
@@ -1238,6 +1246,11 @@ cudaError_t launch_kns(const EncArgs& a, int sm_count, int smem_optin, cudaStrea
       switch (a.L.nsplit) {
         case 1:
           // few waves of chunks: one group per CTA (see MaxThreads)
+          if (a.C == 4096 && a.W == 4096 && a.m == 4 && a.M == 259) {  // the configs' parameters
+            if (a.N < kG1MaxWaves * 9u * (uint32_t)sm_count)
+              return launch_k<4, 1, LZ, true, false, 4096, true>(a, sm_count, smem_optin, s, launches);
+            return launch_k<4, 1, LZ, false, false, 4096, true>(a, sm_count, smem_optin, s, launches);
+          }
           if (a.N < kG1MaxWaves * 9u * (uint32_t)sm_count)
             return a.C == 4096 ? launch_k<4, 1, LZ, true, false, 4096>(a, sm_count, smem_optin, s, launches)
                                : launch_k<4, 1, LZ, true>(a, sm_count, smem_optin, s, launches);
