@@ -152,7 +152,7 @@ __host__ __device__ constexpr EncLayout enc_layout(uint32_t C, uint32_t K, uint3
   // list; ctrl (4 + 2K words)
   L.max_runs = enc_max_runs(C);
   const bool tbg = big || K >= 16;  // walk bitmaps in the global scratch
-  o += 4 * (2 * L.bm_words + (tbg ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K);
+  o += 4 * (2 * L.bm_words + (tbg ? 0 : K * L.tb_words) + L.max_runs + 4 + 2 * K + (C + 1023) / 1024);
   o = align_up(o, 8);
   L.off_mbar = o;
   o += 8;
