@@ -66,10 +66,14 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
 }
 
 
+// CF, MF != 0: specialised for chunk size CF and min match MF (compile-time)
+template <uint32_t CF, uint32_t MF>
 __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_kernel(
     const uint8_t* __restrict__ comp, const uint32_t* __restrict__ sizes,
-    const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C, uint32_t m,
-    uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride, uint64_t err_base) {
+    const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C_in, uint32_t m_in,
+    uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride_in, uint64_t err_base) {
+  const uint32_t C = CF ? CF : C_in, m = MF ? MF : m_in;
+  const uint32_t buf_stride = CF ? align_up(CF, 16) : buf_stride_in;
   extern __shared__ __align__(16) uint8_t dsm[];
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   uint8_t* obuf = dsm + (size_t)warp * buf_stride;  // rebuilt chunk (C bytes)
@@ -283,7 +287,9 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   {
     std::lock_guard<std::mutex> lk(mu);
     if (!cache[dev].attr) {
-      e = cudaFuncSetAttribute(lzr_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
+      e = cudaFuncSetAttribute(lzr_decode_kernel<0, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(lzr_decode_kernel<4096, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
       if (e != cudaSuccess) return e;
       cache[dev].attr = true;
     }
@@ -291,7 +297,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   }
   if (per_sm == 0) {
     // (LZR_DEC_ONEWAVE: at most one resident wave of CTAs, warps loop over chunks)
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel, warps * 32, smem);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, lzr_decode_kernel<0, 0>, warps * 32, smem);
     if (e != cudaSuccess || per_sm < 1) per_sm = 1;
     std::lock_guard<std::mutex> lk(mu);
     cache[dev].smem = smem;
@@ -305,7 +311,11 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
   size_t blocks = (N + warps - 1) / warps;
   const size_t cap = (size_t)sm_count * per_sm;
   if (LZR_DEC_ONEWAVE && blocks > cap) blocks = cap;
-  lzr_decode_kernel<<<(unsigned)blocks, warps * 32, smem, s>>>(comp, sizes, offsets, n_bytes, C, m,
+  if (C == 4096 && m == 4)  // the configs' chunk size and min match
+    lzr_decode_kernel<4096, 4><<<(unsigned)blocks, warps * 32, smem, s>>>(comp, sizes, offsets, n_bytes, C, m,
+                                                                         out, errp, N, stride, err_base);
+  else
+  lzr_decode_kernel<0, 0><<<(unsigned)blocks, warps * 32, smem, s>>>(comp, sizes, offsets, n_bytes, C, m,
                                                               out, errp, N, stride, err_base);
   if (launches) ++*launches;
   e = cudaGetLastError();
