@@ -45,7 +45,7 @@ constexpr int32_t kNoError = 0x7F7F7F7F;
 #ifndef LZR_DEC_LANE_MAX
 #define LZR_DEC_LANE_MAX 16
 #endif
-constexpr uint32_t kLaneCopyMax = LZR_DEC_LANE_MAX;  // matches up to this length: one lane, byte-serial
+constexpr uint32_t kLaneCopyMax = LZR_DEC_LANE_MAX;  // final-sourced matches up to this length: one lane each
 // (measured and not kept, 1 x B200, 256 MiB, output GB/s mix/text/zero-runs:
 // an L1 prefetch of the stream's lines at chunk start 356/247/702 vs
 // 386/247/667; short matches copied 4 source bytes per step from two aligned
@@ -66,6 +66,26 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
 }
 
 
+// shared-memory bytes by 32-bit address (keeps the rebuilt chunk's base in one
+// register; ordered, the copies below rely on program order within a lane)
+__device__ __forceinline__ uint32_t lds8(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts8(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+
+// inclusive prefix sum over the warp (shfl.up's own predicate marks lanes >= delta)
+__device__ __forceinline__ uint32_t warp_incl_sum(uint32_t v) {
+#pragma unroll
+  for (uint32_t o = 1; o < 32; o <<= 1)
+    asm("{\n\t.reg .u32 t;\n\t.reg .pred p;\n\tshfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t@p add.u32 %0, %0, t;\n\t}"
+        : "+r"(v) : "r"(o));
+  return v;
+}
+
 // CF, MF != 0: specialised for chunk size CF and min match MF (compile-time)
 template <uint32_t CF, uint32_t MF>
 __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_kernel(
@@ -80,7 +100,8 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
   const size_t gw = (size_t)blockIdx.x * (blockDim.x >> 5) + warp;
   const size_t nw = (size_t)gridDim.x * (blockDim.x >> 5);
   const uint32_t g = lane >> 3, j = lane & 7u;
-  const uint32_t below = (1u << j) - 1u;
+  const uint32_t below = (1u << j) - 1u, jbit = 1u << j;  // token j's flag bit and the ones before it
+  const uint32_t sbuf = smem_u32(obuf);
   for (size_t c = gw; c < N; c += nw) {
     const size_t lo = c * C;
     const uint32_t n = (uint32_t)min((size_t)C, n_bytes - lo);
@@ -104,117 +125,113 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       continue;
     }
     bool bad = S > n;
-    // A step reads at most 4 groups (<= 100 bytes) from ip.  The 128 stream
-    // bytes from ip (32 aligned words, one per lane: a coalesced load, bytes
-    // outside the stream read as 0) are loaded before the step -- the next
-    // step's window is issued as soon as this step's end is known, so its
-    // latency hides under the match copies -- and the parse takes its bytes
-    // from the window by shuffle instead of a chain of dependent loads.
+    // Stream positions below are in the aligned view src - mis ("x"
+    // coordinates: stream byte i is x = i + mis).  A step reads at most 4
+    // groups (<= 100 bytes) from ip: the 128 bytes from ip's word (one aligned
+    // word per lane, a coalesced load, bytes outside the stream read as 0) are
+    // loaded before the step -- the next step's window is issued as soon as
+    // this step's end is known, so its latency hides under the copies -- and
+    // the parse takes its bytes from the window by shuffle.
     const uint32_t mis = (uint32_t)((uintptr_t)src & 3u);
-    uint32_t ip = 0, op = 0;
-    uint32_t wbase = mis >> 2;  // first word of the window (aligned view src - mis)
-    uint32_t win = bad ? 0u : load_word(src, mis, S, wbase + lane);
+    const uint32_t Sx = S + mis;
+    uint32_t ip = mis, op = 0;
+    uint32_t wbase = 0;  // first word of the window
+    uint32_t win = bad ? 0u : load_word(src, mis, S, lane);
     while (!bad && op < n) {
       const uint32_t wb = wbase, wv = win;
-      auto sb = [&](uint32_t x) -> uint32_t {  // stream byte x (x <= ip + 101), 0 past the end
-        const uint32_t xx = x + mis;
-        return (__shfl_sync(kFull, wv, (xx >> 2) - wb) >> ((xx & 3u) << 3)) & 0xFFu;
+      auto sbyte = [&](uint32_t x) -> uint32_t {  // stream byte at x (x <= ip + 100)
+        return __byte_perm(__shfl_sync(kFull, wv, (x >> 2) - wb), 0u, (x & 3u) | 0x4440u);
       };
-      // the four groups of this step: flag byte and stream offset
-      uint32_t f = 0, ipg = 0;
-      {
-        uint32_t x = ip;
+      // the flag-byte chain: the lanes of group g stop after g hops
+      uint32_t x = ip;
 #pragma unroll
-        for (uint32_t t = 0; t < 4; ++t) {
-          const uint32_t ft = sb(x);
-          if (t == g) {
-            f = ft;
-            ipg = x;
-          }
-          x += 9u + 2u * __popc(ft);
-        }
+      for (uint32_t t = 0; t < 3; ++t) {
+        const uint32_t ft = sbyte(x);
+        if (g > t) x += 9u + 2u * __popc(ft);
       }
-      const uint32_t ism = (f >> j) & 1u;
-      const uint32_t toff = ipg + 1u + j + 2u * __popc(f & below);
-      const uint32_t tsz = 1u + 2u * ism;
+      const uint32_t f = sbyte(x);
+      const bool ism = (f & jbit) != 0u;
+      const uint32_t toff = x + 1u + j + 2u * __popc(f & below);
+      const uint32_t tend = toff + (ism ? 3u : 1u);  // stream position after the token
       // the token's 3 header bytes from the two window words around toff
-      uint32_t b0, b1, b2;
+      uint32_t hv;
       {
-        const uint32_t xx = toff + mis;
-        const uint32_t wi = (xx >> 2) - wb;
-        const uint32_t lo = __shfl_sync(kFull, wv, wi), hi = __shfl_sync(kFull, wv, wi + 1);
-        const uint32_t v = __funnelshift_r(lo, hi, (xx & 3u) << 3);
-        b0 = v & 0xFFu;
-        b1 = ism ? (v >> 8) & 0xFFu : 0u;
-        b2 = ism ? (v >> 16) & 0xFFu : 0u;
+        const uint32_t wi = (toff >> 2) - wb;
+        hv = __funnelshift_r(__shfl_sync(kFull, wv, wi), __shfl_sync(kFull, wv, wi + 1), (toff & 3u) << 3);
       }
-      const uint32_t tlen = ism ? b2 + m : 1u;
-      const uint32_t d = (b0 | (b1 << 8)) + 1u;
-      uint32_t incl = tlen;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(kFull, incl, o);
-        if ((int)lane >= o) incl += t;
-      }
+      const uint32_t tlen = ism ? __byte_perm(hv, 0u, 0x4442u) + m : 1u;
+      const uint32_t d = (hv & 0xFFFFu) + 1u;
+      const uint32_t incl = warp_incl_sum(tlen);
       const uint32_t ob = op + incl - tlen;  // output position of token `lane`
-      // a group is live when the groups before it did not finish the chunk
-      const uint32_t gstart = __shfl_sync(kFull, ob, lane & ~7u);
-      const bool live = gstart < n;
-      const bool reached = live && ob < n;
-      bool e = false;
-      if (live && ipg >= S) e = true;  // flag byte past the stream
-      if (reached) {
-        if (toff + tsz > S) e = true;
-        if (ism && (d > ob || ob + tlen > n)) e = true;
-      } else if (live && ism) {
-        e = true;  // padding flag bits must be zero
-      }
+      // a group is live when the groups before it did not finish the chunk;
+      // a token is reached when it starts below n (ob grows with the lane)
+      const bool live = __shfl_sync(kFull, ob, lane & ~7u) < n;
+      const bool reached = ob < n;
+      // R15: flag byte or token past the stream, d beyond the output, a match
+      // past n or a set padding flag bit (ob >= n => ob + tlen > n)
+      const bool e = live && (x >= Sx || (ism && (d > ob || ob + tlen > n)) || (reached && tend > Sx));
       if (__any_sync(kFull, e)) {
         bad = true;
         break;
       }
-      const uint32_t rmask = __ballot_sync(kFull, reached);  // a prefix of the lanes
-      const uint32_t last = 31u - __clz(rmask);
+      const uint32_t last = 31u - __clz(__ballot_sync(kFull, reached));  // reached: a prefix of the lanes
+      const uint32_t ipn = __shfl_sync(kFull, tend, last);
+      const uint32_t opn = __shfl_sync(kFull, ob + tlen, last);
       {  // the next step's window, issued now
-        const uint32_t ipn = __shfl_sync(kFull, toff + tsz, last);
-        wbase = (ipn + mis) >> 2;
-        win = ipn < S ? load_word(src, mis, S, wbase + lane) : 0u;
+        wbase = ipn >> 2;
+        win = ipn < Sx ? load_word(src, mis, S, wbase + lane) : 0u;
       }
-      if (reached && !ism) obuf[ob] = (uint8_t)b0;
-      __syncwarp();
-      uint32_t pend = __ballot_sync(kFull, reached && ism);
-      // bytes a match needs before its own output (the rest overlaps itself)
-      const uint32_t need_end = ob - d + min(tlen, d);
-      while (pend) {
-        const uint32_t f0 = (uint32_t)(__ffs(pend) - 1);
-        const uint32_t first_ob = __shfl_sync(kFull, ob, f0);
-        const bool mine = (pend >> lane) & 1u;
-        const uint32_t ready = __ballot_sync(kFull, mine && (lane == f0 || need_end <= first_ob));
-        const bool go = (ready >> lane) & 1u;
-        if (go && tlen <= kLaneCopyMax) {
-          for (uint32_t k = 0; k < tlen; ++k) obuf[ob + k] = obuf[ob - d + k];
+      // Output.  Literals are stored by their lanes.  A match whose source
+      // bytes all lie below op (the step's start; overlapping ones d < l only
+      // need [ob - d, ob)) is final-sourced: the short ones copy at once, one
+      // lane each, byte-serially.  The rest -- long matches and matches that
+      // read this step's output -- follow in token order, each by the whole
+      // warp.
+      if (reached && !ism) sts8(sbuf + ob, hv & 0xFFu);
+      const bool rdy = reached && ism && tlen <= kLaneCopyMax && ob - d + min(tlen, d) <= op;
+      if (rdy) {
+        const uint32_t sa = sbuf + ob - d, da = sbuf + ob;
+        uint32_t k = 0;
+        if (d >= 4u) {
+          for (; k + 4u <= tlen; k += 4u) {
+            const uint32_t b0 = lds8(sa + k), b1 = lds8(sa + k + 1u), b2 = lds8(sa + k + 2u), b3 = lds8(sa + k + 3u);
+            sts8(da + k, b0);
+            sts8(da + k + 1u, b1);
+            sts8(da + k + 2u, b2);
+            sts8(da + k + 3u, b3);
+          }
         }
-        uint32_t lng = ready & __ballot_sync(kFull, tlen > kLaneCopyMax);
-        while (lng) {
-          const int jj = __ffs(lng) - 1;
-          lng &= lng - 1;
-          const uint32_t o = __shfl_sync(kFull, ob, jj);
-          const uint32_t dd = __shfl_sync(kFull, d, jj);
-          const uint32_t ll = __shfl_sync(kFull, tlen, jj);
-          if (dd >= ll) {
-            for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + k];
-          } else {
-            for (uint32_t k = lane; k < ll; k += 32) obuf[o + k] = obuf[o - dd + (k % dd)];
+        for (; k < tlen; ++k) sts8(da + k, lds8(sa + k));
+      }
+      uint32_t rest = __ballot_sync(kFull, reached && ism && !rdy);
+      __syncwarp();
+      while (rest) {
+        const uint32_t jj = __ffs(rest) - 1u;
+        rest &= rest - 1u;
+        const uint32_t o = __shfl_sync(kFull, ob, jj);
+        const uint32_t dd = __shfl_sync(kFull, d, jj);
+        const uint32_t ll = __shfl_sync(kFull, tlen, jj);
+        if (dd >= 32u || dd >= ll) {  // a window of 32 never reads its own bytes
+          for (uint32_t k0 = 0; k0 < ll; k0 += 32u) {  // (warp-uniform trip count: the barrier below)
+            const uint32_t k = k0 + lane;
+            if (k < ll) sts8(sbuf + o + k, lds8(sbuf + o - dd + k));
+            __syncwarp();
+          }
+        } else {  // d < 32, overlapping: out[o + k] = out[o - d + k mod d], all below o
+          const uint32_t sb = sbuf + o - dd, adv = 32u % dd;
+          uint32_t r = lane % dd;
+          for (uint32_t k = lane; k < ll; k += 32u) {
+            sts8(sbuf + o + k, lds8(sb + r));
+            r += adv;
+            if (r >= dd) r -= dd;
           }
           __syncwarp();
         }
-        __syncwarp();
-        pend &= ~ready;
       }
-      op = __shfl_sync(kFull, ob + tlen, last);
-      ip = __shfl_sync(kFull, toff + tsz, last);
+      op = opn;
+      ip = ipn;
     }
-    if (!bad && ip != S) bad = true;
+    if (!bad && ip != Sx) bad = true;
     if (bad) {
       if (lane == 0 && err) atomicMin(err, (int32_t)(c + 1 + err_base));
       __syncwarp();
