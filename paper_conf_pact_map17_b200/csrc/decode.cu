@@ -1,28 +1,30 @@
 // decode.cu -- inverse of the encoder (R1, R5, R9): one warp per chunk, 32
 // tokens (four flag-byte groups) per step.
 //
-// The four flag bytes of a step are a short dependent chain (group g + 1
-// starts 9 + 2 popc(f_g) bytes after group g); then lane t owns token t: its
-// stream offset is ip_g + 1 + j + 2 popc(f_g below j), its output position a
-// 32-lane prefix sum of token lengths.  A step's stream bytes come from a
-// 128-byte window held one word per lane (loaded coalesced while the previous
-// step copies, bytes outside [src, src + S) read as 0) by shuffle.  The chunk
-// is rebuilt in shared memory: literals of the step are stored in parallel,
-// then the step's matches are resolved in rounds -- a match whose source bytes
-// lie below the first unresolved match's output (or that is the first one) is
-// final-sourced, so all such matches copy at once: short ones one lane each,
-// byte-serially (which also gives overlapping matches, d < l, their R5
-// meaning), long ones by the whole warp (out[o + k] = out[o - d + (k mod d)]
-// only reads bytes before o).  The chunk is written out with 16-byte stores;
-// raw chunks are copied with 16-byte stores from funnel-shifted 4-byte loads.
+// Parse: the four flag bytes of a step are a short dependent chain (group g + 1
+// starts 9 + 2 popc(f_g) bytes after group g; the lanes of group g stop after
+// g hops); then lane t owns token t: its stream offset is ip_g + 1 + j +
+// 2 popc(f_g below j), its output position a 32-lane prefix sum of token
+// lengths.  A step's stream bytes come from a 128-byte window held one word per
+// lane (loaded coalesced while the previous step copies, bytes outside
+// [src, src + S) read as 0) by shuffle.
+// Output: the chunk is rebuilt in shared memory.  Literals are stored by their
+// lanes.  Matches whose source bytes all lie below the step's start (and that
+// do not overlap themselves) are "final-sourced": they are listed in token
+// order and copied by all 32 lanes at once, each match by 32/P lanes (P = their
+// count rounded up to a power of two), so a step's short copies cost about
+// l/(32/P) iterations instead of max(l).  The rest -- long matches, matches
+// that read this step's output, overlapping ones (d < l, R5) -- follow in token
+// order, each by the whole warp (overlapping: out[o + k] = out[o - d + k mod
+// d], all below o).  The chunk is written out with 16-byte stores; raw chunks
+// are copied with 16-byte stores from funnel-shifted 4-byte loads.
 // Malformed streams set *err = min(1 + chunk index) (err pre-set to 0x7F7F7F7F,
 // fixed up to 0 afterwards when no chunk was corrupt); with err == NULL nothing
 // is reported (include/lzr.h) and the library keeps no global error word.
-// (An output-parallel variant -- each step's output rebuilt in 32-byte windows,
-// lane = byte, token found by a REDUX.OR of the window's token starts, sources
-// by (o - ob) mod d and in-window pointer jumping, stream staged in shared
-// memory -- measured no faster: text 230-248 vs 243 GB/s, zero-runs 318-395 vs
-// 677.)
+// (Replaced and measured: round 1-2's lane-per-match byte-serial
+// copies in dependency rounds -- 23% of the text decode's instructions in the
+// byte loop; output-parallel 32-byte windows, lane = byte, token by an
+// OR-reduction of the window's token starts -- as costly per byte.)
 #include <mutex>
 
 #include "lzr_internal.cuh"
@@ -40,12 +42,15 @@ namespace {
 #define LZR_DEC_MINB 24
 #endif
 constexpr int32_t kNoError = 0x7F7F7F7F;
-// (1 x B200, 256 MiB, mix/text GB/s: 8 -> 347/208, 12 -> 392/241, 16 ->
-// 402/248, 24 -> 404/250; byte-serial copies 4 at a time with d >= 4: 389/234)
+constexpr uint32_t kCopyList = 32 * sizeof(uint2);  // per warp, after its chunk buffer
+// final-sourced matches up to this length go to the lane-spread copy (1 x
+// B200, 256 MiB, output GB/s mix/text/zero-runs: 16 -> 562/362/871, 32 ->
+// 568/367/875, 64 -> 566/366/871; the copy list packs the length in 8 bits)
 #ifndef LZR_DEC_LANE_MAX
-#define LZR_DEC_LANE_MAX 16
+#define LZR_DEC_LANE_MAX 32
 #endif
-constexpr uint32_t kLaneCopyMax = LZR_DEC_LANE_MAX;  // final-sourced matches up to this length: one lane each
+constexpr uint32_t kLaneCopyMax = LZR_DEC_LANE_MAX;
+static_assert(kLaneCopyMax < 256, "copy-list length field");
 // (measured and not kept, 1 x B200, 256 MiB, output GB/s mix/text/zero-runs:
 // an L1 prefetch of the stream's lines at chunk start 356/247/702 vs
 // 386/247/667; short matches copied 4 source bytes per step from two aligned
@@ -77,6 +82,13 @@ __device__ __forceinline__ void sts8(uint32_t a, uint32_t v) {
   asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 
+// byte (x & 3) of w in all four bytes
+__device__ __forceinline__ uint32_t prmt_rc8(uint32_t w, uint32_t x) {
+  uint32_t r;
+  asm("prmt.b32.rc8 %0, %1, 0, %2;" : "=r"(r) : "r"(w), "r"(x));
+  return r;
+}
+
 // inclusive prefix sum over the warp (shfl.up's own predicate marks lanes >= delta)
 __device__ __forceinline__ uint32_t warp_incl_sum(uint32_t v) {
 #pragma unroll
@@ -93,10 +105,12 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
     const uint64_t* __restrict__ offsets, size_t n_bytes, uint32_t C_in, uint32_t m_in,
     uint8_t* __restrict__ out, int32_t* err, size_t N, uint32_t buf_stride_in, uint64_t err_base) {
   const uint32_t C = CF ? CF : C_in, m = MF ? MF : m_in;
-  const uint32_t buf_stride = CF ? align_up(CF, 16) : buf_stride_in;
+  const uint32_t buf_stride = CF ? align_up(CF, 16) + kCopyList : buf_stride_in;
   extern __shared__ __align__(16) uint8_t dsm[];
   const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
   uint8_t* obuf = dsm + (size_t)warp * buf_stride;  // rebuilt chunk (C bytes)
+  // the step's final-sourced matches (source, destination | length << 24)
+  uint2* clist = reinterpret_cast<uint2*>(obuf + buf_stride - kCopyList);
   const size_t gw = (size_t)blockIdx.x * (blockDim.x >> 5) + warp;
   const size_t nw = (size_t)gridDim.x * (blockDim.x >> 5);
   const uint32_t g = lane >> 3, j = lane & 7u;
@@ -139,17 +153,20 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
     uint32_t win = bad ? 0u : load_word(src, mis, S, lane);
     while (!bad && op < n) {
       const uint32_t wb = wbase, wv = win;
-      auto sbyte = [&](uint32_t x) -> uint32_t {  // stream byte at x (x <= ip + 100)
-        return __byte_perm(__shfl_sync(kFull, wv, (x >> 2) - wb), 0u, (x & 3u) | 0x4440u);
+      // stream byte at x (x <= ip + 100) replicated into all four bytes of
+      // the result (prmt.rc8 takes the byte index from x's low bits):
+      // popc(rep) = 4 popc(byte), and rep & mask = byte & mask for masks < 256
+      auto sbyte4 = [&](uint32_t x) -> uint32_t {
+        return prmt_rc8(__shfl_sync(kFull, wv, (x >> 2) - wb), x);
       };
       // the flag-byte chain: the lanes of group g stop after g hops
       uint32_t x = ip;
 #pragma unroll
       for (uint32_t t = 0; t < 3; ++t) {
-        const uint32_t ft = sbyte(x);
-        if (g > t) x += 9u + 2u * __popc(ft);
+        const uint32_t ft = sbyte4(x);
+        if (g > t) x += 9u + (__popc(ft) >> 1);
       }
-      const uint32_t f = sbyte(x);
+      const uint32_t f = sbyte4(x);
       const bool ism = (f & jbit) != 0u;
       const uint32_t toff = x + 1u + j + 2u * __popc(f & below);
       const uint32_t tend = toff + (ism ? 3u : 1u);  // stream position after the token
@@ -165,8 +182,9 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       const uint32_t ob = op + incl - tlen;  // output position of token `lane`
       // a group is live when the groups before it did not finish the chunk;
       // a token is reached when it starts below n (ob grows with the lane)
-      const bool live = __shfl_sync(kFull, ob, lane & ~7u) < n;
       const bool reached = ob < n;
+      const uint32_t rmask = __ballot_sync(kFull, reached);  // a prefix of the lanes
+      const bool live = (rmask >> (lane & ~7u)) & 1u;
       // R15: flag byte or token past the stream, d beyond the output, a match
       // past n or a set padding flag bit (ob >= n => ob + tlen > n)
       const bool e = live && (x >= Sx || (ism && (d > ob || ob + tlen > n)) || (reached && tend > Sx));
@@ -174,7 +192,7 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
         bad = true;
         break;
       }
-      const uint32_t last = 31u - __clz(__ballot_sync(kFull, reached));  // reached: a prefix of the lanes
+      const uint32_t last = 31u - __clz(rmask);
       const uint32_t ipn = __shfl_sync(kFull, tend, last);
       const uint32_t opn = __shfl_sync(kFull, ob + tlen, last);
       {  // the next step's window, issued now
@@ -188,20 +206,23 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       // read this step's output -- follow in token order, each by the whole
       // warp.
       if (reached && !ism) sts8(sbuf + ob, hv & 0xFFu);
-      const bool rdy = reached && ism && tlen <= kLaneCopyMax && ob - d + min(tlen, d) <= op;
-      if (rdy) {
-        const uint32_t sa = sbuf + ob - d, da = sbuf + ob;
-        uint32_t k = 0;
-        if (d >= 4u) {
-          for (; k + 4u <= tlen; k += 4u) {
-            const uint32_t b0 = lds8(sa + k), b1 = lds8(sa + k + 1u), b2 = lds8(sa + k + 2u), b3 = lds8(sa + k + 3u);
-            sts8(da + k, b0);
-            sts8(da + k + 1u, b1);
-            sts8(da + k + 2u, b2);
-            sts8(da + k + 3u, b3);
-          }
+      const bool rdy = reached && ism && tlen <= kLaneCopyMax && d >= tlen && ob - d + tlen <= op;
+      if (reached && !ism) sts8(sbuf + ob, hv & 0xFFu);
+      const uint32_t rset = __ballot_sync(kFull, rdy);
+      if (rset) {
+        // the nr final-sourced matches are listed in token order; lane L
+        // copies bytes h, h + H, ... of match L mod P (P = nr rounded up to
+        // a power of two, h = L / P, H = 32 / P): no byte of them is read by
+        // another (d >= l, sources below op)
+        if (rdy) clist[__popc(rset & lanemask_lt())] = make_uint2(sbuf + ob - d, (sbuf + ob) | (tlen << 24));
+        __syncwarp();
+        const uint32_t nr = __popc(rset), lg = 32u - __clz(nr - 1u);
+        const uint32_t mi = lane & ((1u << lg) - 1u);
+        if (mi < nr) {
+          const uint2 cl = clist[mi];
+          const uint32_t len = cl.y >> 24, da = cl.y & 0xFFFFFFu, step = 32u >> lg;
+          for (uint32_t k = lane >> lg; k < len; k += step) sts8(da + k, lds8(cl.x + k));
         }
-        for (; k < tlen; ++k) sts8(da + k, lds8(sa + k));
       }
       uint32_t rest = __ballot_sync(kFull, reached && ism && !rdy);
       __syncwarp();
@@ -271,7 +292,7 @@ cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint
     if (err && err_own) return cudaMemsetAsync(err, 0, sizeof(int32_t), s);
     return cudaSuccess;
   }
-  const uint32_t stride = align_up(C, 16);  // rebuilt chunk
+  const uint32_t stride = align_up(C, 16) + kCopyList;  // rebuilt chunk + copy list
 // Grid: 2 warps (chunks) per CTA and one CTA per 2 chunks, so the hardware
 // block scheduler balances chunks of very different cost (raw copies vs text)
 // as CTAs retire; a persistent one-wave grid of 16-warp CTAs left SMs idle at
