@@ -1,13 +1,14 @@
-// decode.cu -- inverse of the encoder (R1, R5, R9): one warp per chunk, 32
-// tokens (four flag-byte groups) per step.
+// decode.cu -- inverse of the encoder (R1, R5, R9): one warp per chunk, up to
+// 64 tokens (eight flag-byte groups) per step.
 //
-// Parse: the four flag bytes of a step are a short dependent chain (group g + 1
-// starts 9 + 2 popc(f_g) bytes after group g; the lanes of group g stop after
-// g hops); then lane t owns token t: its stream offset is ip_g + 1 + j +
-// 2 popc(f_g below j), its output position a 32-lane prefix sum of token
-// lengths.  A step's stream bytes come from a 128-byte window held one word per
+// Parse: a step's stream bytes come from a 128-byte window held one word per
 // lane (loaded coalesced while the previous step copies, bytes outside
-// [src, src + S) read as 0) by shuffle.
+// [src, src + S) read as 0) by shuffle; the step takes the groups that lie
+// wholly inside it (text: all eight, most steps).  The flag bytes are a short
+// dependent chain (group g + 1 starts 9 + 2 popc(f_g) bytes after group g; the
+// lanes of group g stop after g hops); lane L owns tokens j0 = 2 (L mod 4) and
+// j0 + 1 of group L / 4: stream offset ip_g + 1 + j0 + 2 popc(f_g below j0),
+// output position a 32-lane prefix sum of the lanes' two token lengths.
 // Output: the chunk is rebuilt in shared memory.  Literals are stored by their
 // lanes.  Matches whose source bytes all lie below the step's start (and that
 // do not overlap themselves) are "final-sourced": they are listed in token
@@ -62,6 +63,7 @@ __device__ __forceinline__ uint32_t load_word(const uint8_t* src, uint32_t mis, 
                                               uint32_t i) {
   const uint32_t b = i << 2;
   if (b >= mis && b + 4 <= mis + len) return __ldg(reinterpret_cast<const uint32_t*>(src - mis) + i);
+  if (b + 4 <= mis || b >= mis + len) return 0u;
   uint32_t v = 0;
   for (uint32_t t = 0; t < 4; ++t) {
     const uint32_t x = b + t;
@@ -113,8 +115,8 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
   uint2* clist = reinterpret_cast<uint2*>(obuf + buf_stride - kCopyList);
   const size_t gw = (size_t)blockIdx.x * (blockDim.x >> 5) + warp;
   const size_t nw = (size_t)gridDim.x * (blockDim.x >> 5);
-  const uint32_t g = lane >> 3, j = lane & 7u;
-  const uint32_t below = (1u << j) - 1u, jbit = 1u << j;  // token j's flag bit and the ones before it
+  const uint32_t g = lane >> 2, j0 = (lane & 3u) << 1;  // tokens j0, j0 + 1 of group g
+  const uint32_t below0 = (1u << j0) - 1u, bit0 = 1u << j0, bit1 = 2u << j0;
   const uint32_t sbuf = smem_u32(obuf);
   for (size_t c = gw; c < N; c += nw) {
     const size_t lo = c * C;
@@ -140,12 +142,11 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
     }
     bool bad = S > n;
     // Stream positions below are in the aligned view src - mis ("x"
-    // coordinates: stream byte i is x = i + mis).  A step reads at most 4
-    // groups (<= 100 bytes) from ip: the 128 bytes from ip's word (one aligned
-    // word per lane, a coalesced load, bytes outside the stream read as 0) are
-    // loaded before the step -- the next step's window is issued as soon as
-    // this step's end is known, so its latency hides under the copies -- and
-    // the parse takes its bytes from the window by shuffle.
+    // coordinates: stream byte i is x = i + mis).  A step parses the groups
+    // (up to 8, 64 tokens) that lie wholly inside a 128-byte window from ip's
+    // word (one aligned word per lane, a coalesced load, bytes outside the
+    // stream read as 0); the next step's window is issued as soon as this
+    // step's end is known, so its latency hides under the copies.
     const uint32_t mis = (uint32_t)((uintptr_t)src & 3u);
     const uint32_t Sx = S + mis;
     uint32_t ip = mis, op = 0;
@@ -153,70 +154,87 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
     uint32_t win = bad ? 0u : load_word(src, mis, S, lane);
     while (!bad && op < n) {
       const uint32_t wb = wbase, wv = win;
-      // stream byte at x (x <= ip + 100) replicated into all four bytes of
-      // the result (prmt.rc8 takes the byte index from x's low bits):
-      // popc(rep) = 4 popc(byte), and rep & mask = byte & mask for masks < 256
+      const uint32_t wend = (wb << 2) + 128u;
+      // stream byte at x replicated into all four bytes (prmt.rc8 takes the
+      // byte index from x's low bits): popc(rep) = 4 popc(byte), and
+      // rep & mask = byte & mask for masks < 256
       auto sbyte4 = [&](uint32_t x) -> uint32_t {
         return prmt_rc8(__shfl_sync(kFull, wv, (x >> 2) - wb), x);
       };
       // the flag-byte chain: the lanes of group g stop after g hops
       uint32_t x = ip;
 #pragma unroll
-      for (uint32_t t = 0; t < 3; ++t) {
+      for (uint32_t t = 0; t < 7; ++t) {
         const uint32_t ft = sbyte4(x);
         if (g > t) x += 9u + (__popc(ft) >> 1);
       }
       const uint32_t f = sbyte4(x);
-      const bool ism = (f & jbit) != 0u;
-      const uint32_t toff = x + 1u + j + 2u * __popc(f & below);
-      const uint32_t tend = toff + (ism ? 3u : 1u);  // stream position after the token
-      // the token's 3 header bytes from the two window words around toff
-      uint32_t hv;
+      // this step takes the groups whose flag byte and 8 token slots lie in
+      // the window (a prefix of the groups; group 0 always fits)
+      const bool fits = x + 9u + (__popc(f) >> 1) <= wend;
+      // tokens 2(lane mod 4) and +1 of group g
+      const bool ism0 = fits && (f & bit0) != 0u, ism1 = fits && (f & bit1) != 0u;
+      const uint32_t toff0 = x + 1u + j0 + 2u * __popc(f & below0);
+      const uint32_t toff1 = toff0 + (ism0 ? 3u : 1u);
+      const uint32_t tend0 = toff1, tend1 = toff1 + (ism1 ? 3u : 1u);
+      // both tokens' header bytes from the three window words from toff0's
+      uint32_t hv0, hv1;
       {
-        const uint32_t wi = (toff >> 2) - wb;
-        hv = __funnelshift_r(__shfl_sync(kFull, wv, wi), __shfl_sync(kFull, wv, wi + 1), (toff & 3u) << 3);
+        const uint32_t wi = (toff0 >> 2) - wb;
+        const uint32_t w0 = __shfl_sync(kFull, wv, wi), w1 = __shfl_sync(kFull, wv, wi + 1u),
+                       w2 = __shfl_sync(kFull, wv, wi + 2u);
+        hv0 = __funnelshift_r(w0, w1, (toff0 & 3u) << 3);
+        const uint32_t r = toff1 - (toff0 & ~3u);  // 1..6
+        hv1 = r < 4u ? __funnelshift_r(w0, w1, r << 3) : __funnelshift_r(w1, w2, (r - 4u) << 3);
       }
-      const uint32_t tlen = ism ? __byte_perm(hv, 0u, 0x4442u) + m : 1u;
-      const uint32_t d = (hv & 0xFFFFu) + 1u;
-      const uint32_t incl = warp_incl_sum(tlen);
-      const uint32_t ob = op + incl - tlen;  // output position of token `lane`
-      // a group is live when the groups before it did not finish the chunk;
-      // a token is reached when it starts below n (ob grows with the lane)
-      const bool reached = ob < n;
-      const uint32_t rmask = __ballot_sync(kFull, reached);  // a prefix of the lanes
-      const bool live = (rmask >> (lane & ~7u)) & 1u;
+      const uint32_t tlen0 = ism0 ? __byte_perm(hv0, 0u, 0x4442u) + m : (fits ? 1u : 0u);
+      const uint32_t tlen1 = ism1 ? __byte_perm(hv1, 0u, 0x4442u) + m : (fits ? 1u : 0u);
+      const uint32_t d0 = (hv0 & 0xFFFFu) + 1u, d1 = (hv1 & 0xFFFFu) + 1u;
+      const uint32_t incl = warp_incl_sum(tlen0 + tlen1);
+      const uint32_t ob0 = op + incl - tlen0 - tlen1, ob1 = ob0 + tlen0;  // output positions
+      // a token is reached when it is parsed and starts below n; a group is
+      // live when its first token is reached
+      const bool reached0 = fits && ob0 < n, reached1 = fits && ob1 < n;
+      const uint32_t rm0 = __ballot_sync(kFull, reached0), rm1 = __ballot_sync(kFull, reached1);
+      const bool live = (rm0 >> (lane & ~3u)) & 1u;
       // R15: flag byte or token past the stream, d beyond the output, a match
       // past n or a set padding flag bit (ob >= n => ob + tlen > n)
-      const bool e = live && (x >= Sx || (ism && (d > ob || ob + tlen > n)) || (reached && tend > Sx));
+      const bool e = live && (x >= Sx || (ism0 && (d0 > ob0 || ob0 + tlen0 > n)) ||
+                              (ism1 && (d1 > ob1 || ob1 + tlen1 > n)) || (reached0 && tend0 > Sx) ||
+                              (reached1 && tend1 > Sx));
       if (__any_sync(kFull, e)) {
         bad = true;
         break;
       }
-      const uint32_t last = 31u - __clz(rmask);
-      const uint32_t ipn = __shfl_sync(kFull, tend, last);
-      const uint32_t opn = __shfl_sync(kFull, ob + tlen, last);
+      // the last reached token: token 1 of lane l0 if reached, else token 0
+      const uint32_t l0 = 31u - __clz(rm0);
+      const uint32_t ipn = __shfl_sync(kFull, reached1 ? tend1 : tend0, l0);
+      const uint32_t opn = __shfl_sync(kFull, reached1 ? ob1 + tlen1 : ob0 + tlen0, l0);
       {  // the next step's window, issued now
         wbase = ipn >> 2;
         win = ipn < Sx ? load_word(src, mis, S, wbase + lane) : 0u;
       }
-      // Output.  Literals are stored by their lanes.  A match whose source
-      // bytes all lie below op (the step's start; overlapping ones d < l only
-      // need [ob - d, ob)) is final-sourced: the short ones copy at once, one
-      // lane each, byte-serially.  The rest -- long matches and matches that
-      // read this step's output -- follow in token order, each by the whole
-      // warp.
-      if (reached && !ism) sts8(sbuf + ob, hv & 0xFFu);
-      const bool rdy = reached && ism && tlen <= kLaneCopyMax && d >= tlen && ob - d + tlen <= op;
-      if (reached && !ism) sts8(sbuf + ob, hv & 0xFFu);
-      const uint32_t rset = __ballot_sync(kFull, rdy);
-      if (rset) {
-        // the nr final-sourced matches are listed in token order; lane L
-        // copies bytes h, h + H, ... of match L mod P (P = nr rounded up to
-        // a power of two, h = L / P, H = 32 / P): no byte of them is read by
-        // another (d >= l, sources below op)
-        if (rdy) clist[__popc(rset & lanemask_lt())] = make_uint2(sbuf + ob - d, (sbuf + ob) | (tlen << 24));
+      // Output.  Literals are stored by their lanes.  Matches whose source
+      // bytes all lie below op and that do not overlap themselves are listed in
+      // token order and copied by all lanes at once; the rest follow in token
+      // order, each by the whole warp.
+      if (reached0 && !ism0) sts8(sbuf + ob0, hv0 & 0xFFu);
+      if (reached1 && !ism1) sts8(sbuf + ob1, hv1 & 0xFFu);
+      bool rdy0 = reached0 && ism0 && tlen0 <= kLaneCopyMax && d0 >= tlen0 && ob0 - d0 + tlen0 <= op;
+      bool rdy1 = reached1 && ism1 && tlen1 <= kLaneCopyMax && d1 >= tlen1 && ob1 - d1 + tlen1 <= op;
+      const uint32_t R0 = __ballot_sync(kFull, rdy0), R1 = __ballot_sync(kFull, rdy1);
+      if (R0 | R1) {
+        // the list holds 32 entries: later ones go to the token-order pass
+        const uint32_t lt = lanemask_lt();
+        const uint32_t rk = __popc(R0 & lt) + __popc(R1 & lt);
+        rdy0 = rdy0 && rk < 32u;
+        rdy1 = rdy1 && rk + rdy0 < 32u;
+        if (rdy0) clist[rk] = make_uint2(sbuf + ob0 - d0, (sbuf + ob0) | (tlen0 << 24));
+        if (rdy1) clist[rk + rdy0] = make_uint2(sbuf + ob1 - d1, (sbuf + ob1) | (tlen1 << 24));
         __syncwarp();
-        const uint32_t nr = __popc(rset), lg = 32u - __clz(nr - 1u);
+        const uint32_t nr = min(__popc(R0) + __popc(R1), 32u), lg = 32u - __clz(nr - 1u);
+        // lane L copies bytes h, h + H, ... of entry L mod P (P = nr rounded
+        // up to a power of two, h = L / P, H = 32 / P)
         const uint32_t mi = lane & ((1u << lg) - 1u);
         if (mi < nr) {
           const uint2 cl = clist[mi];
@@ -224,14 +242,17 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
           for (uint32_t k = lane >> lg; k < len; k += step) sts8(da + k, lds8(cl.x + k));
         }
       }
-      uint32_t rest = __ballot_sync(kFull, reached && ism && !rdy);
+      uint32_t X0 = __ballot_sync(kFull, reached0 && ism0 && !rdy0);
+      uint32_t X1 = __ballot_sync(kFull, reached1 && ism1 && !rdy1);
       __syncwarp();
-      while (rest) {
-        const uint32_t jj = __ffs(rest) - 1u;
-        rest &= rest - 1u;
-        const uint32_t o = __shfl_sync(kFull, ob, jj);
-        const uint32_t dd = __shfl_sync(kFull, d, jj);
-        const uint32_t ll = __shfl_sync(kFull, tlen, jj);
+      while (X0 | X1) {
+        const uint32_t jj = __ffs(X0 | X1) - 1u;
+        const bool second = !((X0 >> jj) & 1u);  // token 1 of lane jj
+        if (second) X1 &= X1 - 1u;
+        else X0 &= ~(1u << jj);
+        const uint32_t o = __shfl_sync(kFull, second ? ob1 : ob0, jj);
+        const uint32_t dd = __shfl_sync(kFull, second ? d1 : d0, jj);
+        const uint32_t ll = __shfl_sync(kFull, second ? tlen1 : tlen0, jj);
         if (dd >= 32u || dd >= ll) {  // a window of 32 never reads its own bytes
           for (uint32_t k0 = 0; k0 < ll; k0 += 32u) {  // (warp-uniform trip count: the barrier below)
             const uint32_t k = k0 + lane;
