@@ -11,10 +11,10 @@
 // output position a 32-lane prefix sum of the lanes' two token lengths.
 // Output: the chunk is rebuilt in shared memory.  Literals are stored by their
 // lanes.  Matches whose source bytes all lie below the step's start (and that
-// do not overlap themselves) are "final-sourced": they are listed in token
-// order and copied by all 32 lanes at once, each match by 32/P lanes (P = their
-// count rounded up to a power of two), so a step's short copies cost about
-// l/(32/P) iterations instead of max(l).  The rest -- long matches, matches
+// do not overlap themselves) are "final-sourced": the first 32 of a step are
+// listed in token order (shared memory) and copied by all 32 lanes at once,
+// each match by 32/P lanes (P = their count rounded up to a power of two), so
+// a step's short copies cost about l/(32/P) iterations instead of max(l).  The rest -- long matches, matches
 // that read this step's output, overlapping ones (d < l, R5) -- follow in token
 // order, each by the whole warp (overlapping: out[o + k] = out[o - d + k mod
 // d], all below o).  The chunk is written out with 16-byte stores; raw chunks
