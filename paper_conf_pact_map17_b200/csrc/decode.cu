@@ -91,6 +91,21 @@ __device__ __forceinline__ uint32_t prmt_rc8(uint32_t w, uint32_t x) {
   return r;
 }
 
+// Debug build (-DLZR_DEC_CHECK, tools/check_decode.sh): every shared-memory
+// access of the rebuild traps unless it stays inside the chunk's bytes and
+// reads only bytes already final (compute-sanitizer is not available on the
+// GPU pool; this is the bounds check that replaces it for the decoder).
+#ifdef LZR_DEC_CHECK
+#define DEC_ASSERT(c) \
+  do {            \
+    if (!(c)) __trap(); \
+  } while (0)
+#else
+#define DEC_ASSERT(c) \
+  do {            \
+  } while (0)
+#endif
+
 // inclusive prefix sum over the warp (shfl.up's own predicate marks lanes >= delta)
 __device__ __forceinline__ uint32_t warp_incl_sum(uint32_t v) {
 #pragma unroll
@@ -218,6 +233,8 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       // bytes all lie below op and that do not overlap themselves are listed in
       // token order and copied by all lanes at once; the rest follow in token
       // order, each by the whole warp.
+      DEC_ASSERT(!(reached0 && !ism0) || ob0 < n);
+      DEC_ASSERT(!(reached1 && !ism1) || ob1 < n);
       if (reached0 && !ism0) sts8(sbuf + ob0, hv0 & 0xFFu);
       if (reached1 && !ism1) sts8(sbuf + ob1, hv1 & 0xFFu);
       bool rdy0 = reached0 && ism0 && tlen0 <= kLaneCopyMax && d0 >= tlen0 && ob0 - d0 + tlen0 <= op;
@@ -239,6 +256,7 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
         if (mi < nr) {
           const uint2 cl = clist[mi];
           const uint32_t len = cl.y >> 24, da = cl.y & 0xFFFFFFu, step = 32u >> lg;
+          DEC_ASSERT(cl.x >= sbuf && cl.x + len <= sbuf + op && da >= sbuf + op && da + len <= sbuf + n);
           for (uint32_t k = lane >> lg; k < len; k += step) sts8(da + k, lds8(cl.x + k));
         }
       }
@@ -256,6 +274,7 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
         if (dd >= 32u || dd >= ll) {  // a window of 32 never reads its own bytes
           for (uint32_t k0 = 0; k0 < ll; k0 += 32u) {  // (warp-uniform trip count: the barrier below)
             const uint32_t k = k0 + lane;
+            DEC_ASSERT(k >= ll || (dd <= o && o + k < n));
             if (k < ll) sts8(sbuf + o + k, lds8(sbuf + o - dd + k));
             __syncwarp();
           }
@@ -263,6 +282,7 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
           const uint32_t sb = sbuf + o - dd, adv = 32u % dd;
           uint32_t r = lane % dd;
           for (uint32_t k = lane; k < ll; k += 32u) {
+            DEC_ASSERT(sb >= sbuf && sb + r < sbuf + o && o + k < n);
             sts8(sbuf + o + k, lds8(sb + r));
             r += adv;
             if (r >= dd) r -= dd;

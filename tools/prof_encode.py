@@ -29,4 +29,6 @@ for _ in range(a.iters):
     if a.decode:
         y, err = lzr.decompress(out, sizes, offs, n, p)
 torch.cuda.synchronize()
-print("total", int(total.item()), "CR", n / int(total.item()))
+if a.decode:  # the round trip must hold (bounds-checked builds run this too)
+    assert int(err.item()) == 0 and torch.equal(y, x), "decode round trip failed"
+print("total", int(total.item()), "CR", n / int(total.item()), "round trip ok" if a.decode else "")
