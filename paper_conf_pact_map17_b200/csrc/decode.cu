@@ -257,7 +257,13 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
           const uint2 cl = clist[mi];
           const uint32_t len = cl.y >> 24, da = cl.y & 0xFFFFFFu, step = 32u >> lg;
           DEC_ASSERT(cl.x >= sbuf && cl.x + len <= sbuf + op && da >= sbuf + op && da + len <= sbuf + n);
-          for (uint32_t k = lane >> lg; k < len; k += step) sts8(da + k, lds8(cl.x + k));
+          uint32_t k = lane >> lg;
+          for (; k + step < len; k += 2u * step) {  // two bytes per iteration
+            const uint32_t b0 = lds8(cl.x + k), b1 = lds8(cl.x + k + step);
+            sts8(da + k, b0);
+            sts8(da + k + step, b1);
+          }
+          if (k < len) sts8(da + k, lds8(cl.x + k));
         }
       }
       uint32_t X0 = __ballot_sync(kFull, reached0 && ism0 && !rdy0);
