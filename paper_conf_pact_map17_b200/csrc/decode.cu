@@ -277,7 +277,11 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
         const uint32_t o = __shfl_sync(kFull, second ? ob1 : ob0, jj);
         const uint32_t dd = __shfl_sync(kFull, second ? d1 : d0, jj);
         const uint32_t ll = __shfl_sync(kFull, second ? tlen1 : tlen0, jj);
-        if (dd >= 32u || dd >= ll) {  // a window of 32 never reads its own bytes
+        if (ll <= 32u && dd >= ll) {  // one window, no loop (most of them)
+          DEC_ASSERT(lane >= ll || (dd <= o && o + lane < n));
+          if (lane < ll) sts8(sbuf + o + lane, lds8(sbuf + o - dd + lane));
+          __syncwarp();
+        } else if (dd >= 32u || dd >= ll) {  // a window of 32 never reads its own bytes
           for (uint32_t k0 = 0; k0 < ll; k0 += 32u) {  // (warp-uniform trip count: the barrier below)
             const uint32_t k = k0 + lane;
             DEC_ASSERT(k >= ll || (dd <= o && o + k < n));
