@@ -1,4 +1,4 @@
-# usage: bash tools/scratch_abn.sh PARITY_VARIANT V1 V2 ...: decode timing of the variants (alternating, 2 rounds), parity tests on the first
+# usage: bash tools/ab_decode.sh PARITY_VARIANT V1 V2 ...: decode timing of the variants (alternating, 2 rounds), parity tests on the first
 P=$1; shift
 for r in 1 2; do for V in "$@"; do
 LZR_LIBRARY=paper_conf_pact_map17_b200/liblzr_$V.so python tools/dec_time.py mix text zeroruns random 2>&1 | tail -1
