@@ -511,3 +511,63 @@ def test_random_params_fuzz(lzr, ref, seed):
     n = int(C * rng.integers(2, 5) + rng.integers(0, C))
     x = synth.fill_host(n, C, cls, seed=seed)
     _check_full(lzr, ref, x, lzr.Params(chunk_size=C, window=W, min_match=m, max_match=M, parse=parse))
+
+
+def _decoder_paths_inputs(C: int, m: int, seed: int):
+    """Chunks built to drive the decoder's step paths (decode.cu): (A) all-match
+    streams of (m + 1)-byte copies from the first quarter -- groups of 25 bytes, so a
+    step takes 5 of its 8 groups, and more than 32 final-sourced matches per
+    step (list overflow into the token-order pass); (B) periodic runs with
+    periods 1..70 (overlapping matches, d < l, both below and above 32);
+    (C) words from a small vocabulary (short matches reading the same step's
+    output: the token-order pass)."""
+    rng = np.random.default_rng(seed)
+    q = C // 4
+    a = []
+    for _ in range(3):
+        head = rng.integers(0, 256, q, dtype=np.uint8)
+        offs = rng.integers(0, q - m - 1, (C - q) // (m + 1) + 1)
+        a.append(np.concatenate([head, np.concatenate([head[o:o + m + 1] for o in offs])])[:C])
+    b = []
+    for _ in range(3):
+        parts, tot = [], 0
+        while tot < C:
+            per = int(rng.integers(1, 71))
+            ln = int(rng.integers(per + 1, per + 300))
+            base = rng.integers(0, 256, per, dtype=np.uint8)
+            parts.append(np.tile(base, ln // per + 1)[:ln])
+            tot += ln
+        b.append(np.concatenate(parts)[:C])
+    vocab = [rng.integers(97, 123, int(rng.integers(3, 8)), dtype=np.uint8) for _ in range(16)]
+    c = []
+    for _ in range(3):
+        parts, tot = [], 0
+        while tot < C:
+            w = vocab[int(rng.integers(0, 16))]
+            parts.append(np.append(w, np.uint8(32)))
+            tot += w.size + 1
+        c.append(np.concatenate(parts)[:C])
+    return np.concatenate(a + b + c + [c[0][: C // 3]])  # + a ragged tail chunk
+
+
+@pytest.mark.parametrize("C,m", [(4096, 4), (4096, 3), (1024, 3), (4096, 6), (65536, 4)])
+def test_decoder_step_paths_vs_oracle(lzr, ref, C, m):
+    """GPU decode of oracle-compressed streams (the two share no code) that
+    drive the decoder's step paths; the first kind must really put > 32 match
+    tokens into one 64-token step."""
+    from tests.lzss_check import parse_stream
+
+    x = _decoder_paths_inputs(C, m, seed=C + m)
+    rp = ref.Params(chunk_size=C, window=C, min_match=m, max_match=m + 255)
+    r_out, r_sizes, r_offs, r_tot = ref.compress(x, rp)
+    if C <= 4096:
+        toks = parse_stream(bytes(r_out[r_offs[1]:r_offs[1] + r_sizes[1]]), C, m)
+        assert max(sum(1 for ln, d in toks[i:i + 64] if d) for i in range(0, len(toks), 64)) > 32
+    p = lzr.Params(chunk_size=C, min_match=m)
+    d_out = torch.from_numpy(r_out).cuda()
+    d_sizes = torch.from_numpy(r_sizes.view(np.int32)).cuda()
+    d_offs = torch.from_numpy(r_offs.view(np.int64)).cuda()
+    y, err = lzr.decompress(d_out, d_sizes, d_offs, x.size, p)
+    torch.cuda.synchronize()
+    assert int(err.item()) == 0
+    assert np.array_equal(y.cpu().numpy(), x)
