@@ -145,8 +145,14 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
       for (uint32_t i = lane * 16; i < n16; i += 32 * 16) {
         const uint32_t w0 = (mis + i) >> 2;
         uint32_t v[5];
+        if (i >= 4u && i + 20u <= n) {  // the five words lie inside the chunk's bytes
+          const uint32_t* sw = reinterpret_cast<const uint32_t*>(src - mis) + w0;
 #pragma unroll
-        for (int t = 0; t < 5; ++t) v[t] = load_word(src, mis, n, w0 + t);
+          for (int t = 0; t < 5; ++t) v[t] = __ldg(sw + t);
+        } else {
+#pragma unroll
+          for (int t = 0; t < 5; ++t) v[t] = load_word(src, mis, n, w0 + t);
+        }
         const uint32_t sh = mis << 3;
         *reinterpret_cast<uint4*>(dst + i) =
             make_uint4(__funnelshift_r(v[0], v[1], sh), __funnelshift_r(v[1], v[2], sh),
