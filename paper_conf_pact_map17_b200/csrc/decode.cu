@@ -295,8 +295,12 @@ __global__ void __launch_bounds__(32 * LZR_DEC_WARPS, LZR_DEC_MINB) lzr_decode_k
             __syncwarp();
           }
         } else {  // d < 32, overlapping: out[o + k] = out[o - d + k mod d], all below o
-          const uint32_t sb = sbuf + o - dd, adv = 32u % dd;
-          uint32_t r = lane % dd;
+          // lane mod d and 32 mod d for d < 32 by a float reciprocal: q = floor((x + 0.5) / d)
+          // is exact for x <= 32, d < 32 (checked for every pair in IEEE single)
+          const float rd = __frcp_rn((float)dd);
+          const uint32_t sb = sbuf + o - dd;
+          const uint32_t adv = 32u - dd * (uint32_t)(32.5f * rd);
+          uint32_t r = lane - dd * (uint32_t)(((float)lane + 0.5f) * rd);
           for (uint32_t k = lane; k < ll; k += 32u) {
             DEC_ASSERT(sb >= sbuf && sb + r < sbuf + o && o + k < n);
             sts8(sbuf + o + k, lds8(sb + r));

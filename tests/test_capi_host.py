@@ -118,3 +118,13 @@ def test_no_gpu_fails_loudly(lzr):
     assert st == lzr.ERR_CUDA
     with pytest.raises(Exception):
         lzr.compress(torch.zeros(4096, dtype=torch.uint8), p)  # CPU tensor: no CPU path
+
+
+def test_decoder_float_mod_identity():
+    """decode.cu's periodic copies take x mod d (x <= 32, 1 <= d < 32) as
+    x - d * floor((x + 0.5) * rcp(d)) in IEEE single precision: exact for every pair."""
+    for d in range(1, 32):
+        rd = np.float32(1.0) / np.float32(d)
+        for x in range(0, 33):
+            q = int(np.float32(np.float32(x) + np.float32(0.5)) * rd)
+            assert q == x // d, (x, d)
