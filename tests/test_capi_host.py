@@ -121,10 +121,10 @@ def test_no_gpu_fails_loudly(lzr):
 
 
 def test_decoder_float_mod_identity():
-    import numpy as np
-
     """decode.cu's periodic copies take x mod d (x <= 32, 1 <= d < 32) as
     x - d * floor((x + 0.5) * rcp(d)) in IEEE single precision: exact for every pair."""
+    import numpy as np
+
     for d in range(1, 32):
         rd = np.float32(1.0) / np.float32(d)
         for x in range(0, 33):
