@@ -25,6 +25,7 @@ thread-per-chunk on the host cores) on a bounded sample of the same workload.
 from __future__ import annotations
 
 import argparse
+import ctypes
 import json
 import os
 import statistics
@@ -553,6 +554,9 @@ def per_class(lzr, synth, p, n, dev, stream, steps=5, warmup=2):
     ws = lzr.Workspace(n, p, dev)
     y = torch.empty(n, dtype=torch.uint8, device=dev)
     err = torch.zeros(1, dtype=torch.int32, device=dev)
+    import ctypes
+    dws = torch.empty(lzr.lib().lzr_decompress_workspace_bytes(n, ctypes.byref(p.c())), dtype=torch.uint8,
+                      device=dev)
     res = {}
     for cls in ("text", "random", "zeroruns"):
         synth.fill_device(x, p.chunk_size, cls)
@@ -564,7 +568,7 @@ def per_class(lzr, synth, p, n, dev, stream, steps=5, warmup=2):
             lzr.compress(x, p, ws=ws)
         e[1].record(stream)
         for _ in range(steps):
-            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n, p, y, err)
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n, p, y, err, workspace=dws)
         e[2].record(stream)
         torch.cuda.synchronize()
         tot = int(ws.total.item())
@@ -781,14 +785,17 @@ def main():
     if not a.no_decode:
         dout = torch.empty(n_rank, dtype=torch.uint8, device=dev)
         derr = torch.zeros(1, dtype=torch.int32, device=dev)
+        # the decode schedule's workspace (chunks costliest first), allocated once
+        dws = torch.empty(lzr.lib().lzr_decompress_workspace_bytes(n_rank, ctypes.byref(p.c())),
+                          dtype=torch.uint8, device=dev)
         for _ in range(a.warmup):
-            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr, workspace=dws)
         d0, d1e = mk(), mk()
         torch.cuda.synchronize()
         R.barrier()
         d0.record(stream)
         for _ in range(a.steps):
-            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr)
+            lzr.decompress(ws.out, ws.sizes[: ws.N], ws.offsets[: ws.N], n_rank, p, dout, derr, workspace=dws)
         d1e.record(stream)
         torch.cuda.synchronize()
         dms = R.reduce(d0.elapsed_time(d1e) / a.steps, "max")

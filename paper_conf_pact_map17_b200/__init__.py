@@ -33,7 +33,7 @@ PARSE_GREEDY, PARSE_LAZY = 0, 1  # lzr_params.parse (include/lzr.h; R8
 EXPORTED_SYMBOLS = [
     "lzr_validate_params", "lzr_num_chunks", "lzr_compress_bound", "lzr_compress_workspace_bytes",
     "lzr_compress_chunks", "lzr_compress_encode", "lzr_compress_compact",
-    "lzr_scan_workspace_bytes", "lzr_scan_sizes", "lzr_decompress_chunks",
+    "lzr_scan_workspace_bytes", "lzr_scan_sizes", "lzr_decompress_workspace_bytes", "lzr_decompress_chunks",
     "lzr_compress_host_scratch_bytes", "lzr_compress_host", "lzr_status_str",
     "lzr_last_launch_count", "lzr_fingerprint_chunks", "lzr_dedup_table_bytes", "lzr_dedup_index",
     "lzr_gather_chunks", "lzr_dedup_index_gidx", "lzr_dedup_owner_counts", "lzr_dedup_route",
@@ -96,7 +96,9 @@ def lib():
         L.lzr_scan_workspace_bytes.argtypes = [sz]
         L.lzr_scan_workspace_bytes.restype = sz
         L.lzr_scan_sizes.argtypes = [vp, sz, u64, vp, vp, vp, sz, vp]
-        L.lzr_decompress_chunks.argtypes = [vp, vp, vp, sz, P, vp, vp, vp]
+        L.lzr_decompress_workspace_bytes.argtypes = [sz, P]
+        L.lzr_decompress_workspace_bytes.restype = sz
+        L.lzr_decompress_chunks.argtypes = [vp, vp, vp, sz, P, vp, vp, vp, sz, vp]
         L.lzr_compress_host_scratch_bytes.argtypes = [sz, P]
         L.lzr_compress_host_scratch_bytes.restype = sz
         L.lzr_compress_host.argtypes = [vp, sz, P, vp, sz, vp, vp, vp, sz, vp, sz]
@@ -273,9 +275,12 @@ def scan_sizes(sizes, base: int = 0, offsets=None, total=None, ws=None, stream=N
 
 
 def decompress(comp, sizes, offsets, n: int, p: Params = Params(), out=None, error=None,
-               stream=None):
+               stream=None, workspace=None, schedule: bool = True):
     """Decode chunk streams back into n bytes.  Returns (out, error) where
-    error is an int32[1] device tensor: 0 or 1 + index of the first corrupt chunk."""
+    error is an int32[1] device tensor: 0 or 1 + index of the first corrupt chunk.
+    schedule: decode the chunks costliest first (needs a workspace of
+    lzr_decompress_workspace_bytes; allocated here when not given); the
+    output is the same either way."""
     import torch
 
     dev = comp.device
@@ -284,9 +289,17 @@ def decompress(comp, sizes, offsets, n: int, p: Params = Params(), out=None, err
             out = torch.empty(max(1, n), dtype=torch.uint8, device=dev)
         if error is None:
             error = torch.zeros(1, dtype=torch.int32, device=dev)
+        ws_bytes = 0
+        if schedule:
+            ws_bytes = lib().lzr_decompress_workspace_bytes(n, ctypes.byref(p.c()))
+            if workspace is None:
+                workspace = torch.empty(max(1, ws_bytes), dtype=torch.uint8, device=dev)
+            _same_device(comp, workspace)
+            ws_bytes = workspace.numel()
         _same_device(comp, sizes, offsets, out, error)
         st = lib().lzr_decompress_chunks(_ptr(comp), _ptr(sizes), _ptr(offsets), n,
                                          ctypes.byref(p.c()), _ptr(out), _ptr(error),
+                                         _ptr(workspace) if schedule else None, ws_bytes,
                                          _stream(stream, dev))
     _check(st, "lzr_decompress_chunks")
     return out[:n], error

@@ -388,9 +388,15 @@ int lzr_gather_chunks(const void* d_in, size_t n_bytes, uint32_t chunk_size,
   return LZR_OK;
 }
 
+size_t lzr_decompress_workspace_bytes(size_t n_bytes, const lzr_params* p) {
+  if (lzr_validate_params(p) != LZR_OK) return 0;
+  const size_t C = p->chunk_size;
+  return align_up_z(decode_sched_bytes((n_bytes + C - 1) / C), 256);
+}
+
 int lzr_decompress_chunks(const void* d_comp, const uint32_t* d_sizes, const uint64_t* d_offsets,
                           size_t n_bytes, const lzr_params* p, void* d_out, int32_t* d_error,
-                          lzr_stream_t stream) {
+                          void* d_workspace, size_t workspace_bytes, lzr_stream_t stream) {
   t_launches = 0;
   int st = lzr_validate_params(p);
   if (st) return st;
@@ -402,9 +408,15 @@ int lzr_decompress_chunks(const void* d_comp, const uint32_t* d_sizes, const uin
   if (dev_info(&di) != cudaSuccess) return LZR_ERR_CUDA;
   if ((int)align_up(p->chunk_size, 16) > di.smem_optin)
     return LZR_ERR_UNSUPPORTED;
+  uint32_t* sched = nullptr;  // the costliest-first schedule needs the workspace
+  if (d_workspace) {
+    if (!aligned(d_workspace, 4)) return LZR_ERR_INVALID_ARG;
+    if (workspace_bytes < lzr_decompress_workspace_bytes(n_bytes, p)) return LZR_ERR_CAPACITY;
+    sched = (uint32_t*)d_workspace;
+  }
   if (launch_decode((const uint8_t*)d_comp, d_sizes, d_offsets, n_bytes, p->chunk_size,
                     p->min_match, (uint8_t*)d_out, d_error, di.sm_count, di.smem_optin, s,
-                    &t_launches) != cudaSuccess)
+                    &t_launches, 0, true, sched) != cudaSuccess)
     return LZR_ERR_CUDA;
   return LZR_OK;
 }
@@ -680,13 +692,15 @@ struct DecSet {
   uint8_t *comp, *out;
   uint32_t* sizes;
   uint64_t* offs;
+  uint32_t* sched;  // the batch's decode schedule
   int32_t* err;
 };
 
 size_t dec_set_bytes(size_t batch, const lzr_params* p) {
   const size_t C = p->chunk_size;
   const size_t N = (batch + C - 1) / C;
-  return 2 * align_up_z(batch, 256) + align_up_z(4 * N, 256) + align_up_z(8 * N, 256) + 256;
+  return 2 * align_up_z(batch, 256) + align_up_z(4 * N, 256) + align_up_z(8 * N, 256) +
+         align_up_z(decode_sched_bytes(N), 256) + 256;
 }
 
 DecSet dec_carve(uint8_t* base, size_t batch, const lzr_params* p) {
@@ -698,6 +712,7 @@ DecSet dec_carve(uint8_t* base, size_t batch, const lzr_params* p) {
   d.out = base + o; o += align_up_z(batch, 256);
   d.sizes = (uint32_t*)(base + o); o += align_up_z(4 * N, 256);
   d.offs = (uint64_t*)(base + o); o += align_up_z(8 * N, 256);
+  d.sched = (uint32_t*)(base + o); o += align_up_z(decode_sched_bytes(N), 256);
   d.err = (int32_t*)(base + o);
   return d;
 }
@@ -777,7 +792,7 @@ int lzr_decompress_host(const void* h_comp, const uint32_t* h_sizes, const uint6
     // offsets are the stream's own: the batch buffer stands at offset lo
     int l = 0;
     if (launch_decode(d.comp - lo, d.sizes, d.offs, len, (uint32_t)C, p->min_match, d.out, derr,
-                      di.sm_count, di.smem_optin, ss, &l, c0, false) != cudaSuccess ||
+                      di.sm_count, di.smem_optin, ss, &l, c0, false, d.sched) != cudaSuccess ||
         cudaEventRecord(hs->ev_kdone[k], ss) != cudaSuccess || cudaStreamWaitEvent(d2h, hs->ev_kdone[k], 0) != cudaSuccess ||
         cudaMemcpyAsync((uint8_t*)h_out + b * batch_bytes, d.out, len, cudaMemcpyDeviceToHost, d2h) != cudaSuccess ||
         cudaEventRecord(hs->ev_out[k], d2h) != cudaSuccess) {

@@ -206,7 +206,9 @@ cudaError_t launch_compact(const uint8_t* in, size_t n_bytes, uint32_t C, const 
 cudaError_t launch_decode(const uint8_t* comp, const uint32_t* sizes, const uint64_t* offsets,
                           size_t n_bytes, uint32_t C, uint32_t m, uint8_t* out, int32_t* err,
                           int sm_count, int smem_optin, cudaStream_t s, int* launches,
-                          uint64_t err_base = 0, bool err_own = true);
+                          uint64_t err_base = 0, bool err_own = true, uint32_t* sched = nullptr);
+// decode schedule workspace (costliest chunks first): 128 counters + N indices
+inline size_t decode_sched_bytes(size_t N) { return (128 + N) * sizeof(uint32_t); }
 cudaError_t decode_err_init(int32_t* err, cudaStream_t s);
 cudaError_t decode_err_fini(int32_t* err, cudaStream_t s, int* launches);
 

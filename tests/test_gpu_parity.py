@@ -453,7 +453,7 @@ def test_decode_without_error_word(lzr):
     y = torch.empty_like(xd)
     st = lzr.lib().lzr_decompress_chunks(
         lzr._ptr(out), lzr._ptr(sizes), lzr._ptr(offs), x.size, ctypes.byref(p.c()), lzr._ptr(y),
-        ctypes.c_void_p(0), ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+        ctypes.c_void_p(0), ctypes.c_void_p(0), 0, ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
     assert st == 0
     torch.cuda.synchronize()
     assert torch.equal(y, xd)
@@ -567,7 +567,39 @@ def test_decoder_step_paths_vs_oracle(lzr, ref, C, m):
     d_out = torch.from_numpy(r_out).cuda()
     d_sizes = torch.from_numpy(r_sizes.view(np.int32)).cuda()
     d_offs = torch.from_numpy(r_offs.view(np.int64)).cuda()
-    y, err = lzr.decompress(d_out, d_sizes, d_offs, x.size, p)
-    torch.cuda.synchronize()
-    assert int(err.item()) == 0
-    assert np.array_equal(y.cpu().numpy(), x)
+    for sched in (True, False):  # costliest-first schedule and index order
+        y, err = lzr.decompress(d_out, d_sizes, d_offs, x.size, p, schedule=sched)
+        torch.cuda.synchronize()
+        assert int(err.item()) == 0
+        assert np.array_equal(y.cpu().numpy(), x)
+
+
+def test_decode_schedule_workspace_and_order(lzr, ref):
+    """The decode schedule: too small a workspace is LZR_ERR_CAPACITY; with and
+    without a workspace the output and the first-corrupt-chunk verdict agree
+    (the schedule changes the order chunks are decoded in, not the result)."""
+    import ctypes
+
+    x = synth.fill_host(64 * 4096 + 999, 4096, "mix", seed=21)
+    p = lzr.Params()
+    xd, out, sizes, offs, tot, g_out, g_sizes, g_offs = _gpu_compress(lzr, x, p)
+    need = lzr.lib().lzr_decompress_workspace_bytes(x.size, ctypes.byref(p.c()))
+    assert need >= 4 * (128 + 65)
+    small = torch.empty(need - 4, dtype=torch.uint8, device="cuda")
+    with pytest.raises(lzr.LzrError):
+        lzr.decompress(out, sizes, offs, x.size, p, workspace=small)
+    for sched in (True, False):
+        y, err = lzr.decompress(out, sizes, offs, x.size, p, schedule=sched)
+        torch.cuda.synchronize()
+        assert int(err.item()) == 0 and torch.equal(y, xd)
+    # two corrupt chunks: the lower index is reported whichever is decoded first
+    bad = g_out.copy()
+    for ci in (40, 9):
+        if g_sizes[ci] < 4096:
+            bad[g_offs[ci] + 1] ^= 0xFF
+    st, r_bad, _ = ref.decompress(bad, g_sizes, g_offs, x.size, ref.Params())
+    d_bad = torch.from_numpy(bad).cuda()
+    for sched in (True, False):
+        _, err = lzr.decompress(d_bad, sizes, offs, x.size, p, schedule=sched)
+        torch.cuda.synchronize()
+        assert int(err.item()) == r_bad
