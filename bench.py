@@ -554,7 +554,6 @@ def per_class(lzr, synth, p, n, dev, stream, steps=5, warmup=2):
     ws = lzr.Workspace(n, p, dev)
     y = torch.empty(n, dtype=torch.uint8, device=dev)
     err = torch.zeros(1, dtype=torch.int32, device=dev)
-    import ctypes
     dws = torch.empty(lzr.lib().lzr_decompress_workspace_bytes(n, ctypes.byref(p.c())), dtype=torch.uint8,
                       device=dev)
     res = {}
@@ -808,7 +807,6 @@ def main():
 
     # ---- end to end through the C ABI with host buffers (pinned), every rank
     if not a.no_e2e:
-        import ctypes
 
         n_e2e = min(n_rank, 1 << 30)  # bounded host buffers for the big configs
         hx = x[:n_e2e].cpu().pin_memory()
