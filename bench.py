@@ -807,7 +807,6 @@ def main():
 
     # ---- end to end through the C ABI with host buffers (pinned), every rank
     if not a.no_e2e:
-
         n_e2e = min(n_rank, 1 << 30)  # bounded host buffers for the big configs
         hx = x[:n_e2e].cpu().pin_memory()
         scratch = torch.empty(max(256, lzr.lib().lzr_compress_host_scratch_bytes(

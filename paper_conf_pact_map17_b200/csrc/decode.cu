@@ -19,6 +19,9 @@
 // order, each by the whole warp (overlapping: out[o + k] = out[o - d + k mod
 // d], all below o).  The chunk is written out with 16-byte stores; raw chunks
 // are copied with 16-byte stores from funnel-shifted 4-byte loads.
+// Schedule: given a workspace, the chunks are decoded costliest first (raw
+// last, compressed ones by size; a bucket sort of the sizes, below), so the
+// end of the grid runs short chunks and a CTA's two chunks cost about the same.
 // Malformed streams set *err = min(1 + chunk index) (err pre-set to 0x7F7F7F7F,
 // fixed up to 0 afterwards when no chunk was corrupt); with err == NULL nothing
 // is reported (include/lzr.h) and the library keeps no global error word.
