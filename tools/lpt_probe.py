@@ -36,3 +36,26 @@ def t(inp, reps=10):
 for r in range(2):
     a, b = t(x), t(xp)
     print(f"as generated {a:.3f} ms ({n / a / 1e6:.1f} GB/s)   costly-first {b:.3f} ms ({n / b / 1e6:.1f} GB/s)")
+
+# the same for the decoder (index order, no schedule): decompression of the two compressed streams
+oa, sa, fa, ta = lzr.compress(x, p)
+ob, sb, fb, tb = lzr.compress(xp, p)
+y = torch.empty_like(x)
+
+
+def td(o, s_, f, reps=10):
+    for _ in range(3):
+        lzr.decompress(o, s_, f, n, p, out=y, schedule=False)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record()
+    for _ in range(reps):
+        lzr.decompress(o, s_, f, n, p, out=y, schedule=False)
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+for r in range(2):
+    a, b = td(oa, sa, fa), td(ob, sb, fb)
+    print(f"decode: as generated {a:.3f} ms ({n / a / 1e6:.1f} GB/s)   costly-first {b:.3f} ms ({n / b / 1e6:.1f} GB/s)")
